@@ -1,0 +1,410 @@
+#!/usr/bin/env python
+"""Benchmark: HGEMM TFLOP/s at M=N=K=8192 on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl ours|reference]
+
+One "step" = one hgemm() call (the whole hot path: TMA staging, tcgen05 MMA
+into TMEM, alpha/beta epilogue) over one batch of synthetic input.
+  N = 1 : the metric configuration, C(8192x8192) = A^T B, FP16 in, FP32
+          accumulate, FP16 out (BASELINE.json configs[1], paper layout TN).
+  N > 1 : torchrun, one rank per GPU; weak scaling: each rank owns one
+          8192-column slab of C (global n = 8192*N) and A is replicated by
+          an NCCL broadcast (timed and reported separately, "collective").
+Timing: W untimed warm-up steps, then K steps, each bracketed by CUDA events
+on the launching stream; L2 is flushed (a 256 MiB write) between steps,
+outside the events; a barrier + synchronize bracket the timed region; the
+time is the max over ranks.  Rank 0 prints ONE JSON line.
+
+--impl reference runs the CPU oracle (oracle/, the correctness reference;
+there is no runnable reference implementation of the paper) on the host
+cores, on a bounded sample of the same workload, and prints the same JSON
+line with "impl": "reference".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "HGEMM TFLOP/s at M=N=K=8192 and % of B200 dense FP16 peak; 1/2/4/8-GPU"
+UNIT = "TFLOP/s"
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return {"tflops_burst": d["bf16_tflops"], "tflops_sustained": d.get("bf16_tflops_sustained"),
+                "hbm_gbs": d["hbm_gbs"], "source": "measured (MEASURED_PEAKS.json; fp16 = bf16 x 1.0 nominal ratio)"}
+    return {"tflops_burst": 1590.0, "tflops_sustained": 1400.0, "hbm_gbs": 6650.0,
+            "source": "fallback (B200_PROFILING.md)"}
+
+
+def load_traffic(workload):
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(workload)
+    return None
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """Samples SM clock and throttle reasons during the timed region (nvidia-smi, else NVML)."""
+
+    def __init__(self, index=0):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _nvml_loop(self):
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            names = {
+                "hw_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwSlowdown", 0x8),
+                "hw_thermal_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
+                "sw_thermal_slowdown": getattr(pynvml, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
+                "sw_power_cap": getattr(pynvml, "nvmlClocksEventReasonSwPowerCap", 0x4),
+                "hw_power_brake_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
+            }
+            while not self._stop.is_set():
+                sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+                try:
+                    rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                except Exception:
+                    rs = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+                self.samples.append((sm, mx, [k for k, v in names.items() if rs & v]))
+                time.sleep(0.05)
+        except Exception as e:  # pragma: no cover
+            self.samples.append((None, None, [f"nvml-error:{type(e).__name__}"]))
+
+    def start(self):
+        self._t = threading.Thread(target=self._nvml_loop, daemon=True)
+        self._t.start()
+
+    def stop(self):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=2)
+        sm = [s[0] for s in self.samples if s[0]]
+        reasons = sorted({r for s in self.samples for r in s[2]})
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max((s[1] for s in self.samples if s[1]), default=None),
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ distributed
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def max_over_ranks(x, world):
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+# ------------------------------------------------------------------ reference arm (oracle)
+def run_reference(args, world, rank):
+    if rank != 0:
+        return 0
+    import numpy as np
+    import oracle
+    from paper_conf_ipps_00020c20_b200 import inputs
+    oracle.build()
+    m, n, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[args.workload]
+    sa = inputs.stored_shape(m, k, tA)
+    sb = inputs.stored_shape(k, n, tB)
+    A = inputs.uniform_f16(sa[0], sa[1], 1).reshape(-1, order="F")
+    B = inputs.uniform_f16(sb[0], sb[1], 2).reshape(-1, order="F")
+    C = (inputs.uniform_f16(m, n, 3).reshape(-1, order="F") if beta != 0 else None)
+    threads = oracle.max_threads()
+    cols = max(1, min(n, args.ref_cols))
+    # sample: `cols` full columns of C (all m rows), each entry a k-long FP64 dot product
+    ii = np.tile(np.arange(m, dtype=np.int64), cols)
+    jj = np.repeat(np.arange(cols, dtype=np.int64), m)
+    times = []
+    for s in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        oracle.hgemm_ref_entries(m, n, k, alpha, A, sa[0], B, sb[0], beta, C, m, tA, tB, out, ii, jj,
+                                 nthreads=threads)
+        dt = time.perf_counter() - t0
+        if s >= args.warmup:
+            times.append(dt)
+    flops = 2.0 * m * cols * k
+    ms = 1e3 * statistics.mean(times)
+    val = flops / (ms * 1e-3) / 1e12
+    sample = f"{cols} full column(s) of C ({m} x {cols} entries, k={k}) of the {m}x{n}x{k} workload per step"
+    line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": args.workload, "m": m, "n": n, "k": k, "layout": tA + tB, "out": out},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def cpu_baseline(workload, budget_s=12.0):
+    """The oracle, as it stands, on the host cores over a bounded sample of the workload."""
+    import numpy as np
+    import oracle
+    from paper_conf_ipps_00020c20_b200 import inputs
+    oracle.build()
+    m, n, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[workload]
+    sa = inputs.stored_shape(m, k, tA)
+    sb = inputs.stored_shape(k, n, tB)
+    A = inputs.uniform_f16(sa[0], sa[1], 1).reshape(-1, order="F")
+    B = inputs.uniform_f16(sb[0], sb[1], 2).reshape(-1, order="F")
+    C = inputs.uniform_f16(m, n, 3).reshape(-1, order="F") if beta != 0 else None
+    threads = oracle.max_threads()
+    # calibrate on a small sample, then size the timed sample to ~budget_s
+    cnt = 4096
+    g = np.random.Generator(np.random.PCG64(0))
+    ii = g.integers(0, m, cnt)
+    jj = g.integers(0, n, cnt)
+    t0 = time.perf_counter()
+    oracle.hgemm_ref_entries(m, n, k, alpha, A, sa[0], B, sb[0], beta, C, m, tA, tB, out, ii, jj, nthreads=threads)
+    dt = max(time.perf_counter() - t0, 1e-4)
+    cnt = int(min(m * n, max(cnt, cnt * budget_s / dt)))
+    ii = g.integers(0, m, cnt)
+    jj = g.integers(0, n, cnt)
+    t0 = time.perf_counter()
+    oracle.hgemm_ref_entries(m, n, k, alpha, A, sa[0], B, sb[0], beta, C, m, tA, tB, out, ii, jj, nthreads=threads)
+    dt = time.perf_counter() - t0
+    return {"value": 2.0 * cnt * k / dt / 1e12, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"{cnt} random entries of C (k={k} FP64 dot products each) of {workload}, {dt:.1f} s"}
+
+
+# ------------------------------------------------------------------ our arm
+def run_ours(args, world, rank, local):
+    import torch
+    from paper_conf_ipps_00020c20_b200 import binding, inputs
+    from paper_conf_ipps_00020c20_b200.sharded import slab_offsets
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    lib = binding.load_library()
+    m, n_rank, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[args.workload]
+    if args.kernel != "auto":
+        binding.set_config(args.kernel, block_n=args.block_n, group_m=args.group_m)
+    elif args.group_m:
+        binding.set_config("auto", group_m=args.group_m)
+    n_glob = n_rank * world
+    n0 = rank * n_rank
+    out_t = torch.float32 if out == "f32" else torch.float16
+    esz = 4 if out == "f32" else 2
+    sa = inputs.stored_shape(m, k, tA)
+    sb_rank = inputs.stored_shape(k, n_rank, tB)
+    # device inputs, seeded on the device (bench-only large configs)
+    g = torch.Generator(device=dev).manual_seed(1234)
+    A = (torch.rand(sa[1], sa[0], generator=g, device=dev) * 2 - 1).half()         # column-major storage
+    gb = torch.Generator(device=dev).manual_seed(5678 + rank)
+    Bs = (torch.rand(sb_rank[1], sb_rank[0], generator=gb, device=dev) * 2 - 1).half()
+    C = torch.zeros(n_rank, m, dtype=out_t, device=dev)                                # slab, column-major
+    if beta != 0:
+        C.uniform_(-1, 1)
+    lda, ldb = sa[0], sb_rank[0]
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+
+    # collective: replicate A (rank 0's copy) over NCCL, timed separately
+    coll = None
+    if world > 1:
+        import torch.distributed as dist
+        for _ in range(2):
+            dist.broadcast(A, src=0)
+        torch.cuda.synchronize()
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        dist.broadcast(A, src=0)
+        e1.record()
+        torch.cuda.synchronize()
+        bms = max_over_ranks(e0.elapsed_time(e1), world)
+        coll = {"op": "broadcast(A) over NCCL", "bytes": A.numel() * 2, "ms": bms,
+                "GB_s": A.numel() * 2 / (bms * 1e-3) / 1e9}
+
+    def step():
+        binding.hgemm(m, n_rank, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out, stream.cuda_stream)
+
+    for _ in range(args.warmup):
+        flush.zero_()
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    launches0 = lib.hgemm_launch_count()
+    clocks = ClockSampler(local)
+    clocks.start()
+    evs = []
+    for _ in range(args.steps):
+        flush.zero_()                                   # L2 flush, outside the events
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        step()
+        e1.record(stream)
+        evs.append((e0, e1))
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    launches = lib.hgemm_launch_count() - launches0
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    ms_local = statistics.mean(step_ms)
+    ms = max_over_ranks(ms_local, world)
+    flops_rank = 2.0 * m * n_rank * k
+    value = flops_rank * world / (ms * 1e-3) / 1e12
+    peaks = load_peaks()
+    achieved = flops_rank / (ms_local * 1e-3) / 1e12
+    stats = binding.get_stats()
+
+    # e2e through the public API with host buffers (pinned), copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        hA = A.cpu().pin_memory()
+        hB = Bs.cpu().pin_memory()
+        hC = torch.empty_like(C, device="cpu").pin_memory()
+        dA2, dB2 = torch.empty_like(A), torch.empty_like(Bs)
+        e2e_steps = max(1, min(args.steps, 10))
+        for it in range(1 + e2e_steps):
+            if it == 1:
+                torch.cuda.synchronize()
+                e0 = torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+            dA2.copy_(hA, non_blocking=True)
+            dB2.copy_(hB, non_blocking=True)
+            binding.hgemm(m, n_rank, k, alpha, dA2, lda, dB2, ldb, beta, C, m, tA, tB, out, stream.cuda_stream)
+            hC.copy_(C, non_blocking=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = max_over_ranks(e0.elapsed_time(e1) / e2e_steps, world)
+        e2e = {"value": flops_rank * world / (ems * 1e-3) / 1e12, "unit": UNIT,
+               "h2d_bytes_per_step": (A.numel() + Bs.numel()) * 2 * world,
+               "d2h_bytes_per_step": C.numel() * esz * world, "ms_per_step": ems}
+
+    # cuBLAS on the same box, same tensors and layout (reference point, north_star (5))
+    cublas = None
+    if not args.no_cublas and rank == 0:
+        try:
+            torch.backends.cuda.matmul.allow_fp16_reduced_precision_reduction = False
+            # Storage tensors are the transposes of the column-major matrices:
+            # A.shape == (cols, rows) of the stored A, so op(A) = A ('T') or A.t() ('N');
+            # likewise op(B) = Bs.t() ('N') or Bs ('T').  Column-major C (m x n) is the
+            # row-major (n x m) tensor C^T = op(B)^T op(A)^T.
+            opA = A if tA in ("T", "t") else A.t()
+            opB = Bs.t() if tB in ("N", "n") else Bs
+            X, Y = opB.t(), opA.t()
+
+            def cub():
+                if out_t == torch.float16:
+                    return torch.mm(X, Y)
+                return torch.mm(X, Y, out_dtype=torch.float32)
+            ref_c = cub()
+            for _ in range(3):
+                cub()
+            torch.cuda.synchronize()
+            ts = []
+            for _ in range(max(3, min(args.steps, 20))):
+                flush.zero_()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                cub()
+                e1.record()
+                ts.append((e0, e1))
+            torch.cuda.synchronize()
+            # agreement with our C (both FP32-accumulated; loose sanity bound only)
+            diff = (ref_c.float() - C.float()).abs().max().item() if beta == 0 else None
+            cms = statistics.mean(a.elapsed_time(b) for a, b in ts)
+            cublas = {"value": flops_rank / (cms * 1e-3) / 1e12, "unit": UNIT, "ms": cms, "max_abs_diff_vs_ours": diff,
+                      "what": "torch.mm (cuBLAS), same operands and layout, fp16 reduced-precision reduction off"}
+        except Exception as e:  # pragma: no cover
+            cublas = {"error": f"{type(e).__name__}: {e}"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(args.workload, budget_s=args.cpu_budget)
+
+    if rank == 0:
+        peak = peaks["tflops_burst"]
+        traffic = load_traffic(args.workload)
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f16xf16->f32 (" + out + " out)", "data": "synthetic",
+            "config": {"workload": args.workload, "m": m, "n": n_glob, "k": k, "n_per_gpu": n_rank,
+                       "layout": tA + tB, "alpha": alpha, "beta": beta, "out": out,
+                       "kernel": stats, "l2": "flushed between steps (256 MiB write, outside the events)",
+                       "parallelism": f"n-slab x{world}" if world > 1 else "single GPU"},
+            "pct_of_peak": 100.0 * value / world / peak,
+            "roofline": {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": UNIT,
+                         "frac": achieved / peak, "traffic": traffic,
+                         "peak_source": peaks["source"] + " burst (kernel timed alone)",
+                         "algorithmic": f"2*m*n*k = {flops_rank:.4e} FLOP per launch"},
+            "gpu_launches": int(launches),
+            "clocks": clk,
+            "e2e": e2e,
+            "cublas": cublas,
+            "cpu_baseline": cpu,
+            "collective": coll,
+            "step_ms": {"min": min(step_ms), "median": statistics.median(step_ms), "max": max(step_ms)},
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="cfg2_8192_TN_f16")
+    ap.add_argument("--kernel", default="auto", choices=["auto", "tc1", "tc2", "simt"])
+    ap.add_argument("--block-n", type=int, default=0)
+    ap.add_argument("--group-m", type=int, default=0)
+    ap.add_argument("--ref-cols", type=int, default=2)
+    ap.add_argument("--cpu-budget", type=float, default=12.0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cublas", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    world, rank, local = dist_env()
+    if args.impl == "reference":
+        return run_reference(args, world, rank)
+    return run_ours(args, world, rank, local)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,111 @@
+/*
+ * include/hgemm.h -- C ABI of the B200-native (sm_100a) half-precision GEMM.
+ *
+ * Operation (SII-A, "C = alpha*A*B + beta*C"; FP16 inputs,
+ * P:401; accumulation in FP32 and FP16 or FP32 output per BASELINE.json
+ * north_star (1)):
+ *
+ *      C <- alpha * op(A) * op(B) + beta * C
+ *
+ * Storage is COLUMN-MAJOR with BLAS/cuBLAS semantics (readings R1,
+ * R2: the paper's "A m x k, B n x k, A row-major, B column-major" benchmark
+ * layout, is transA='T', transB='N' here):
+ *   op(A) is m x k:  transA 'N' -> A is m x k, lda >= max(1,m)
+ *                    transA 'T' -> A is k x m, lda >= max(1,k)
+ *   op(B) is k x n:  transB 'N' -> B is k x n, ldb >= max(1,k)
+ *                    transB 'T' -> B is n x k, ldb >= max(1,n)
+ *   C is m x n, ldc >= max(1,m); element (i,j) at C[i + j*ldc].
+ * A and B hold IEEE binary16 values (__half).  C holds __half when
+ * out_dtype == HGEMM_OUT_F16 and float when HGEMM_OUT_F32; it is read (when
+ * beta != 0) and written in that same type.  Products are accumulated in
+ * FP32 on the tensor cores; the epilogue computes alpha*acc + beta*c in FP32
+ * and rounds once to the output type (round-to-nearest-even, overflow to inf).
+ *
+ * Ownership and lifetime: A, B and C are DEVICE pointers owned by the
+ * caller, who keeps them alive until the work enqueued on `stream`
+ * completes.  The library allocates nothing on the call path and keeps no
+ * pointer after returning.  C must not overlap A or B.
+ *
+ * Asynchrony and errors: hgemm() enqueues on `stream` (0 = legacy default
+ * stream) and returns without synchronising.  Argument errors are detected
+ * synchronously: the call returns HGEMM_ERR_INVALID_VALUE, enqueues nothing
+ * and leaves C untouched.  Launch/encode failures return HGEMM_ERR_CUDA with
+ * the CUDA error left readable by cudaGetLastError().  Device faults surface
+ * at the caller's next synchronisation, as for any CUDA kernel.
+ *
+ * BLAS quick returns: m == 0 or n == 0 -> no-op.  k == 0 or alpha == 0 ->
+ * C = beta*C.  beta == 0 -> C is never read (NaN/Inf in C do not propagate).
+ *
+ * Fast path (tcgen05 tensor cores + TMA): A and B 16-byte aligned, lda and
+ * ldb multiples of 8 elements, C 16-byte aligned and ldc*sizeof(out) a
+ * multiple of 16 bytes.  Anything else runs a slower CUDA-core kernel with
+ * the same semantics (never an error).  All indexing is 64-bit.
+ *
+ * Thread safety: hgemm() is reentrant; per-device properties are cached.
+ * hgemm_set_config() is process-global and meant for tests and benchmarks.
+ */
+#ifndef HGEMM_H_
+#define HGEMM_H_
+
+#include <stdint.h>
+#include <cuda_runtime_api.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum { HGEMM_OUT_F16 = 0, HGEMM_OUT_F32 = 1 } hgemm_dtype_t;
+
+typedef enum {
+    HGEMM_SUCCESS = 0,
+    HGEMM_ERR_INVALID_VALUE = 1, /* m,n,k < 0; bad trans char; ld too small;
+                                    NULL pointer with a nonzero extent; bad out_dtype */
+    HGEMM_ERR_ARCH = 2,          /* current device is not compute capability 10.0 */
+    HGEMM_ERR_CUDA = 3           /* CUDA runtime/driver failure (launch, tensor-map encode) */
+} hgemm_status_t;
+
+/* C <- alpha*op(A)*op(B) + beta*C (see above).  transA/transB in {'N','n','T','t'}. */
+hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k,
+                     float alpha, const void *A, int64_t lda,
+                     const void *B, int64_t ldb,
+                     float beta, void *C, int64_t ldc,
+                     char transA, char transB, hgemm_dtype_t out_dtype,
+                     cudaStream_t stream);
+
+/* Static, NUL-terminated description of a status code (never NULL). */
+const char *hgemm_status_string(hgemm_status_t s);
+
+/* Kernel selection, for tests and benchmarks.  0 fields mean "automatic". */
+typedef enum {
+    HGEMM_KERNEL_AUTO = 0,
+    HGEMM_KERNEL_SIMT = 1,       /* CUDA-core fallback (always available) */
+    HGEMM_KERNEL_TC_1SM = 2,     /* tcgen05 cta_group::1, tile 128 x block_n */
+    HGEMM_KERNEL_TC_2SM = 3      /* tcgen05 cta_group::2 (CTA pair), tile 256 x block_n */
+} hgemm_kernel_t;
+
+typedef struct {
+    int32_t kernel;    /* hgemm_kernel_t */
+    int32_t block_n;   /* tile width along the output's contiguous dim: 64, 128 or 256 (0 = auto) */
+    int32_t group_m;   /* L2 raster group height in tiles (0 = auto) */
+    int32_t max_ctas;  /* cap on persistent CTAs (0 = all SMs) */
+} hgemm_config_t;
+
+/* Set (cfg != NULL) or reset to automatic (cfg == NULL) the process-global
+ * selection.  Returns HGEMM_ERR_INVALID_VALUE for an unknown kernel or
+ * block_n.  A forced tensor-core kernel whose preconditions do not hold
+ * still falls back to SIMT. */
+hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg);
+
+/* The configuration used by the most recent successful hgemm() call in
+ * this process (kernel == HGEMM_KERNEL_AUTO if none, or if it was a quick
+ * return).  `out` must not be NULL. */
+hgemm_status_t hgemm_get_last_config(hgemm_config_t *out);
+
+/* Number of kernel launches hgemm() has enqueued in this process. */
+int64_t hgemm_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* HGEMM_H_ */

@@ -1,0 +1,337 @@
+// Host runtime behind the C ABI of include/hgemm.h: argument validation,
+// BLAS quick returns, kernel selection, TMA tensor-map encoding and launch.
+//
+// Mapping of the column-major ABI onto the kernel (hgemm_tc.cuh):
+//   D = C^T (row-major, ldd = ldc), M = n, N = m,
+//   Ak = op(B)^T  (n x k): transB 'N' -> K-major rows of B; 'T' -> MN-major
+//   Bk = op(A)    (m x k): transA 'T' -> K-major rows of A; 'N' -> MN-major
+// The paper's benchmark layout (A row-major, B column-major)
+// is transA = 'T', transB = 'N': both operands K-major.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdint>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+
+#include "../../include/hgemm.h"
+#include "hgemm_simt.cuh"
+#include "hgemm_tc.cuh"
+
+namespace {
+
+using hg::TcParams;
+using hg::TcShape;
+
+// ----------------------------------------------------------------- device info
+struct DeviceInfo {
+  bool init = false;
+  bool ok = false;
+  int num_sms = 0;
+  int max_clusters_2sm = 0;  // filled lazily per kernel (same for all 2-SM instantiations)
+};
+constexpr int kMaxDevices = 64;
+DeviceInfo g_dev[kMaxDevices];
+std::mutex g_mu;
+
+hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+std::atomic<int64_t> g_launches{0};
+
+bool device_info(int dev, DeviceInfo &out) {
+  if (dev < 0 || dev >= kMaxDevices) return false;
+  std::lock_guard<std::mutex> lk(g_mu);
+  DeviceInfo &d = g_dev[dev];
+  if (!d.init) {
+    int major = 0, minor = 0, sms = 0;
+    if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess ||
+        cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev) != cudaSuccess ||
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+      return false;
+    }
+    d.ok = (major == 10 && minor == 0);
+    d.num_sms = sms;
+    d.init = true;
+  }
+  out = d;
+  return true;
+}
+
+// ----------------------------------------------------------------- tensor maps
+using EncodeTiledFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                   const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &p, 12000, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess) {
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+    }
+  });
+  return fn;
+}
+
+// 2-D FP16 tensor: `inner` contiguous elements per line, `outer` lines `ld` elements apart.
+bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer, int64_t ld, uint32_t box_inner,
+              uint32_t box_outer) {
+  EncodeTiledFn fn = encode_fn();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {static_cast<cuuint64_t>(ld) * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+// ----------------------------------------------------------------- TC launch
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32>
+hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const TcParams &p, int dev,
+                         const DeviceInfo &di, int max_ctas, cudaStream_t stream) {
+  using S = TcShape<BN, CG>;
+  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32>;
+  static int attr_done[kMaxDevices] = {};
+  static int max_clusters[kMaxDevices] = {};
+  if (!attr_done[dev]) {
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, S::SMEM_BYTES) != cudaSuccess)
+      return HGEMM_ERR_CUDA;
+    if (CG == 2) {
+      cudaLaunchConfig_t qc = {};
+      qc.gridDim = dim3(2 * (di.num_sms / 2));
+      qc.blockDim = dim3(192);
+      qc.dynamicSmemBytes = S::SMEM_BYTES;
+      cudaLaunchAttribute qa[1];
+      qa[0].id = cudaLaunchAttributeClusterDimension;
+      qa[0].val.clusterDim.x = 2;
+      qa[0].val.clusterDim.y = 1;
+      qa[0].val.clusterDim.z = 1;
+      qc.attrs = qa;
+      qc.numAttrs = 1;
+      int n = 0;
+      if (cudaOccupancyMaxActiveClusters(&n, kern, &qc) != cudaSuccess || n <= 0) n = di.num_sms / 2;
+      max_clusters[dev] = n;
+    } else {
+      max_clusters[dev] = di.num_sms;
+    }
+    attr_done[dev] = 1;
+  }
+  const int tiles = p.num_m_tiles * p.num_n_tiles;
+  int units = max_clusters[dev];
+  if (max_ctas > 0) units = std::max(1, std::min(units, max_ctas / CG));
+  const int clusters = std::min(tiles, units);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(clusters * CG);
+  cfg.blockDim = dim3(192);
+  cfg.dynamicSmemBytes = S::SMEM_BYTES;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = CG;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (cudaLaunchKernelEx(&cfg, kern, ta, tb, p) != cudaSuccess) return HGEMM_ERR_CUDA;
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+  return HGEMM_SUCCESS;
+}
+
+template <int BN, int CG>
+hgemm_status_t dispatch_tc_layout(bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
+                                  const TcParams &p, int dev, const DeviceInfo &di, int max_ctas, cudaStream_t s) {
+#define HG_CASE(AM, BM_, F)                                                               \
+  if (a_mn == AM && b_mn == BM_ && f32 == F)                                              \
+    return launch_tc<BN, CG, AM, BM_, F>(ta, tb, p, dev, di, max_ctas, s);
+  HG_CASE(false, false, false)
+  HG_CASE(false, false, true)
+  HG_CASE(false, true, false)
+  HG_CASE(false, true, true)
+  HG_CASE(true, false, false)
+  HG_CASE(true, false, true)
+  HG_CASE(true, true, false)
+  HG_CASE(true, true, true)
+#undef HG_CASE
+  return HGEMM_ERR_INVALID_VALUE;
+}
+
+inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+inline bool is_t(char c) { return c == 'T' || c == 't'; }
+inline bool is_n(char c) { return c == 'N' || c == 'n'; }
+inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+// Automatic tile choice: estimated time = waves * per-wave tile cost.
+void choose_tc(int64_t M, int64_t N, int num_sms, int &cg, int &bn) {
+  struct Cand { int cg, bn; double eff; };
+  // eff: relative per-SM throughput of the tile shape (2-SM 256x256 halves
+  // the L2->SM operand traffic per FLOP; 128x128 needs 1.5x the bytes/FLOP of 128x256).
+  const Cand cands[3] = {{2, 256, 1.00}, {1, 256, 0.93}, {1, 128, 0.80}};
+  double best = 1e300;
+  for (const Cand &c : cands) {
+    const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, c.bn);
+    const int64_t units = num_sms / c.cg;
+    const int64_t waves = cdiv(tiles, units);
+    const double t = static_cast<double>(waves) * (128.0 * c.cg * c.bn) / (c.cg * c.eff);
+    if (t < best * 0.999) { best = t; cg = c.cg; bn = c.bn; }
+  }
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *hgemm_status_string(hgemm_status_t s) {
+  switch (s) {
+    case HGEMM_SUCCESS: return "HGEMM_SUCCESS";
+    case HGEMM_ERR_INVALID_VALUE: return "HGEMM_ERR_INVALID_VALUE: invalid argument";
+    case HGEMM_ERR_ARCH: return "HGEMM_ERR_ARCH: device is not compute capability 10.0 (sm_100a)";
+    case HGEMM_ERR_CUDA: return "HGEMM_ERR_CUDA: CUDA runtime/driver error";
+  }
+  return "HGEMM: unknown status";
+}
+
+hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (!cfg) {
+    g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+    return HGEMM_SUCCESS;
+  }
+  if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_TC_2SM) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->block_n != 0 && cfg->block_n != 128 && cfg->block_n != 256) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->kernel == HGEMM_KERNEL_TC_2SM && cfg->block_n == 128) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->group_m < 0 || cfg->max_ctas < 0) return HGEMM_ERR_INVALID_VALUE;
+  g_cfg = *cfg;
+  return HGEMM_SUCCESS;
+}
+
+hgemm_status_t hgemm_get_last_config(hgemm_config_t *out) {
+  if (!out) return HGEMM_ERR_INVALID_VALUE;
+  std::lock_guard<std::mutex> lk(g_mu);
+  *out = g_last;
+  return HGEMM_SUCCESS;
+}
+
+int64_t hgemm_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
+
+hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A, int64_t lda, const void *B,
+                     int64_t ldb, float beta, void *C, int64_t ldc, char transA, char transB,
+                     hgemm_dtype_t out_dtype, cudaStream_t stream) {
+  // ---------------------------------------------------------- validation (no side effects)
+  if (m < 0 || n < 0 || k < 0) return HGEMM_ERR_INVALID_VALUE;
+  if (!(is_t(transA) || is_n(transA)) || !(is_t(transB) || is_n(transB))) return HGEMM_ERR_INVALID_VALUE;
+  if (out_dtype != HGEMM_OUT_F16 && out_dtype != HGEMM_OUT_F32) return HGEMM_ERR_INVALID_VALUE;
+  const bool tA = is_t(transA), tB = is_t(transB);
+  if (lda < std::max<int64_t>(1, tA ? k : m)) return HGEMM_ERR_INVALID_VALUE;
+  if (ldb < std::max<int64_t>(1, tB ? n : k)) return HGEMM_ERR_INVALID_VALUE;
+  if (ldc < std::max<int64_t>(1, m)) return HGEMM_ERR_INVALID_VALUE;
+  if (m == 0 || n == 0) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+    return HGEMM_SUCCESS;
+  }
+  if (!C) return HGEMM_ERR_INVALID_VALUE;
+  const bool need_ab = (k > 0 && alpha != 0.0f);
+  if (need_ab && (!A || !B)) return HGEMM_ERR_INVALID_VALUE;
+
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return HGEMM_ERR_CUDA;
+  DeviceInfo di;
+  if (!device_info(dev, di)) return HGEMM_ERR_CUDA;
+  if (!di.ok) return HGEMM_ERR_ARCH;
+  const bool f32 = (out_dtype == HGEMM_OUT_F32);
+  hgemm_config_t cfg;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    cfg = g_cfg;
+  }
+
+  // ---------------------------------------------------------- BLAS quick return: C = beta*C
+  if (!need_ab) {
+    const int64_t total = m * n;
+    const int threads = 256;
+    const int64_t blocks = std::min<int64_t>(cdiv(total, threads), static_cast<int64_t>(di.num_sms) * 8);
+    if (f32) hg::hgemm_scale_kernel<true><<<static_cast<unsigned>(blocks), threads, 0, stream>>>(m, n, beta, C, ldc);
+    else hg::hgemm_scale_kernel<false><<<static_cast<unsigned>(blocks), threads, 0, stream>>>(m, n, beta, C, ldc);
+    if (cudaPeekAtLastError() != cudaSuccess) return HGEMM_ERR_CUDA;
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+    return HGEMM_SUCCESS;
+  }
+
+  // ---------------------------------------------------------- fast-path preconditions
+  const int out_size = f32 ? 4 : 2;
+  const bool tc_ok = aligned16(A) && aligned16(B) && aligned16(C) && (lda % 8 == 0) && (ldb % 8 == 0) &&
+                     ((ldc * out_size) % 16 == 0) && m < (1ll << 31) && n < (1ll << 31) && k < (1ll << 31) &&
+                     lda < (1ll << 36) && ldb < (1ll << 36) && ldc < (1ll << 36) && encode_fn() != nullptr;
+  const bool want_simt = (cfg.kernel == HGEMM_KERNEL_SIMT);
+  if (!tc_ok || want_simt) {
+    dim3 grid(static_cast<unsigned>(cdiv(m, 64)), static_cast<unsigned>(cdiv(n, 64)));
+    if (grid.y > 65535u) return HGEMM_ERR_INVALID_VALUE;
+    const __half *Ah = static_cast<const __half *>(A);
+    const __half *Bh = static_cast<const __half *>(B);
+    if (f32) hg::hgemm_simt_kernel<true><<<grid, 256, 0, stream>>>(m, n, k, alpha, Ah, lda, Bh, ldb, beta, C, ldc, tA, tB);
+    else hg::hgemm_simt_kernel<false><<<grid, 256, 0, stream>>>(m, n, k, alpha, Ah, lda, Bh, ldb, beta, C, ldc, tA, tB);
+    if (cudaPeekAtLastError() != cudaSuccess) return HGEMM_ERR_CUDA;
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_last = {HGEMM_KERNEL_SIMT, 0, 0, 0};
+    return HGEMM_SUCCESS;
+  }
+
+  // ---------------------------------------------------------- tcgen05 path
+  const int64_t M = n, N = m;  // kernel coordinates (D = C^T)
+  int cg = 2, bn = 256;
+  if (cfg.kernel == HGEMM_KERNEL_TC_1SM) { cg = 1; bn = cfg.block_n ? cfg.block_n : 256; }
+  else if (cfg.kernel == HGEMM_KERNEL_TC_2SM) { cg = 2; bn = 256; }
+  else choose_tc(M, N, di.num_sms, cg, bn);
+  const int bn_cta = bn / cg;
+
+  const bool a_mn = tB;   // Ak = op(B)^T: 'T' -> rows of Ak contiguous along M
+  const bool b_mn = !tA;  // Bk = op(A):   'N' -> rows of Bk contiguous along N
+  CUtensorMap ta, tb;
+  bool ok;
+  if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
+  else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
+  if (ok) {
+    if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, bn_cta);
+    else ok = make_map(&tb, A, static_cast<uint64_t>(m), static_cast<uint64_t>(k), lda, 64, 64);
+  }
+  if (!ok) return HGEMM_ERR_CUDA;
+
+  TcParams p;
+  p.M = static_cast<int32_t>(M);
+  p.N = static_cast<int32_t>(N);
+  p.K = static_cast<int32_t>(k);
+  p.num_m_tiles = static_cast<int32_t>(cdiv(M, 128 * cg));
+  p.num_n_tiles = static_cast<int32_t>(cdiv(N, bn));
+  p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
+  p.group_m = cfg.group_m > 0 ? cfg.group_m : 8;
+  p.group_m = std::max(1, std::min(p.group_m, p.num_m_tiles));
+  p.alpha = alpha;
+  p.beta = beta;
+  p.D = C;
+  p.ldd = ldc;
+
+  hgemm_status_t st;
+  if (cg == 2) st = dispatch_tc_layout<256, 2>(a_mn, b_mn, f32, ta, tb, p, dev, di, cfg.max_ctas, stream);
+  else if (bn == 256) st = dispatch_tc_layout<256, 1>(a_mn, b_mn, f32, ta, tb, p, dev, di, cfg.max_ctas, stream);
+  else st = dispatch_tc_layout<128, 1>(a_mn, b_mn, f32, ta, tb, p, dev, di, cfg.max_ctas, stream);
+  if (st == HGEMM_SUCCESS) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas};
+  }
+  return st;
+}
+
+}  // extern "C"

@@ -1,0 +1,120 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration bench.py
+times (automatic kernel selection), on sampled outputs the oracle computes one
+by one: random entries plus full rows and columns at tile edges."""
+import numpy as np
+import pytest
+
+from paper_conf_ipps_00020c20_b200 import inputs
+
+from .gpu_util import tolerance
+
+pytestmark = pytest.mark.gpu
+
+
+def _device_inputs(m, n, k, tA, tB, seed, beta, out):
+    """Seeded inputs generated on the host (inputs.py) and copied to the device."""
+    import torch
+    sa = inputs.stored_shape(m, k, tA)
+    sb = inputs.stored_shape(k, n, tB)
+    A = inputs.uniform_f16(sa[0], sa[1], seed)          # stored matrices (column-major, ld = rows)
+    B = inputs.uniform_f16(sb[0], sb[1], seed + 1)
+    C = inputs.uniform_f16(m, n, seed + 2) if beta != 0 else None
+    cdt = np.float32 if out == "f32" else np.float16
+    hA = A.reshape(-1, order="F")
+    hB = B.reshape(-1, order="F")
+    hC = (C.astype(cdt).reshape(-1, order="F") if C is not None else np.zeros(m * n, cdt))
+    dA = torch.from_numpy(hA.view(np.int16)).cuda()
+    dB = torch.from_numpy(hB.view(np.int16)).cuda()
+    dC = torch.from_numpy(hC.view(np.int16) if out == "f16" else hC).cuda()
+    return (hA, sa[0]), (hB, sb[0]), hC, dA, dB, dC
+
+
+def _sample_indices(m, n, tile=256, count=4096, seed=0):
+    g = np.random.Generator(np.random.PCG64(seed))
+    ii = list(g.integers(0, m, count))
+    jj = list(g.integers(0, n, count))
+    edge_rows = sorted({0, min(127, m - 1), min(128, m - 1), min(tile - 1, m - 1), min(tile, m - 1), m - 1})
+    edge_cols = sorted({0, min(127, n - 1), min(128, n - 1), min(tile - 1, n - 1), min(tile, n - 1), n - 1})
+    for i in edge_rows:                     # full rows at tile edges
+        ii += [i] * n
+        jj += list(range(n))
+    for j in edge_cols:                     # full columns at tile edges
+        ii += list(range(m))
+        jj += [j] * m
+    return np.array(ii, np.int64), np.array(jj, np.int64)
+
+
+def _check_sampled(oracle_mod, m, n, k, tA, tB, alpha, beta, out, seed=100):
+    import torch
+    from paper_conf_ipps_00020c20_b200 import binding
+    (hA, lda), (hB, ldb), hC, dA, dB, dC = _device_inputs(m, n, k, tA, tB, seed, beta, out)
+    binding.set_config()
+    binding.hgemm(m, n, k, alpha, dA, lda, dB, ldb, beta, dC, m, tA, tB, out)
+    torch.cuda.synchronize()
+    got = dC.cpu().numpy()
+    if out == "f16":
+        got = got.view(np.float16)
+    ii, jj = _sample_indices(m, n, seed=seed)
+    _, r, ab = oracle_mod.hgemm_ref_entries(m, n, k, alpha, hA, lda, hB, ldb, beta, hC, m, tA, tB, out, ii, jj,
+                                            nthreads=oracle_mod.max_threads())
+    g = got[ii + jj * m].astype(np.float64)
+    cvals = hC[ii + jj * m].astype(np.float64) if beta != 0 else None
+    bound = tolerance(r, ab, alpha, beta, cvals, out, g)
+    bad = ~(np.abs(g - r) <= bound)
+    assert not bad.any(), f"{bad.sum()} sampled entries out of tolerance"
+    rel = float(np.max(np.abs(g - r) / np.maximum(ab, 1e-30)))
+    assert rel < 1e-5, rel
+    return got, binding.get_stats()
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("tA,tB,out", [("T", "N", "f16"), ("N", "N", "f16"), ("N", "T", "f16"), ("T", "N", "f32")])
+def test_metric_config_8192(oracle_mod, tA, tB, out):
+    got, stats = _check_sampled(oracle_mod, 8192, 8192, 8192, tA, tB, 1.0, 0.0, out)
+    assert stats["last_kernel"] == "tc2"
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["cfg1_256_NN_f32", "cfg3_bert_ffn1_4096", "cfg3_bert_ffn2_4096",
+                                  "cfg3_lstm_b64", "cfg3_lstm_b256", "cfg3_lstm_b1024", "cfg4_skinny_n64",
+                                  "cfg4_skinny_n128", "cfg4_skinny_n256"])
+def test_baseline_configs(oracle_mod, name):
+    m, n, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[name]
+    _check_sampled(oracle_mod, m, n, k, tA, tB, alpha, beta, out, seed=200)
+
+
+@pytest.mark.slow
+def test_vs_cublas_full_matrix():
+    """Whole-matrix cross-check against cuBLAS (torch.mm, FP32 accumulation forced)."""
+    import torch
+    from paper_conf_ipps_00020c20_b200 import hgemm_torch
+    torch.backends.cuda.matmul.allow_fp16_reduced_precision_reduction = False
+    g = torch.Generator(device="cuda").manual_seed(5)
+    A = (torch.rand(4096, 4096, generator=g, device="cuda") * 2 - 1).half()
+    W = (torch.rand(4096, 4096, generator=g, device="cuda") * 2 - 1).half()
+    ours = hgemm_torch(A, W.t(), out_dtype=torch.float32)
+    ref = torch.mm(A.float(), W.float().t())
+    absab = torch.mm(A.float().abs(), W.float().abs().t())
+    assert torch.all((ours - ref).abs() <= 2e-3 * absab)
+
+
+def test_hgemm_torch_layouts(oracle_mod):
+    import torch
+    from paper_conf_ipps_00020c20_b200 import hgemm_torch
+    M, N, K = 333, 517, 264
+    a = inputs.uniform_f16(M, K, 1)
+    b = inputs.uniform_f16(K, N, 2)
+    exact = a.astype(np.float64) @ b.astype(np.float64)
+    absab = np.abs(a.astype(np.float64)) @ np.abs(b.astype(np.float64))
+    A = torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    B = torch.from_numpy(np.ascontiguousarray(b)).cuda()
+    for Aop in (A, A.t().contiguous().t()):
+        for Bop in (B, B.t().contiguous().t()):
+            C = hgemm_torch(Aop, Bop, out_dtype=torch.float32)
+            assert np.all(np.abs(C.cpu().numpy() - exact) <= 1e-3 * absab)
+    C0 = torch.from_numpy(inputs.uniform_f16(M, N, 3)).cuda()
+    C = C0.clone()
+    hgemm_torch(A, B, C, alpha=0.5, beta=2.0)
+    want = 0.5 * exact + 2.0 * C0.double().cpu().numpy()
+    bound = 1e-3 * (0.5 * absab + 2 * np.abs(C0.double().cpu().numpy())) + 2.0**-9 * np.abs(want) + 2**-24
+    assert np.all(np.abs(C.double().cpu().numpy() - want) <= bound)

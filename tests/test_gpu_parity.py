@@ -1,0 +1,201 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Rules (BASELINE.json north_star (4)):
+  * random inputs in [-1,1): |C_gpu - r| <= 1e-3*(|alpha||A||B| + |beta||C|)_ij,
+    + one FP16 ulp for FP16 output;
+  * integer-valued, identity, permutation and accumulator-width inputs:
+    bit-exact in value (IEEE ==);
+  * beta == 0 never reads C; quick returns; ld padding never read/written.
+Shapes span several tiles plus ragged tails in every dimension.
+"""
+import numpy as np
+import pytest
+
+from paper_conf_ipps_00020c20_b200 import inputs
+
+from .gpu_util import GpuCase, assert_within_tolerance
+
+pytestmark = pytest.mark.gpu
+
+TRANS = [("N", "N"), ("N", "T"), ("T", "N"), ("T", "T")]
+KERNELS = [("tc2", 0), ("tc1", 256), ("tc1", 128), ("simt", 0)]
+
+
+@pytest.fixture(autouse=True)
+def _reset_config():
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config()
+    yield
+    binding.set_config()
+
+
+def _use(kernel, bn):
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config(kernel, block_n=bn)
+
+
+def _expect_kernel(case, kernel):
+    if kernel != "auto":
+        assert case.stats["last_kernel"] == kernel, case.stats
+
+
+@pytest.mark.parametrize("kernel,bn", KERNELS)
+@pytest.mark.parametrize("tA,tB", TRANS)
+@pytest.mark.parametrize("out", ["f16", "f32"])
+def test_random_ragged(oracle_mod, kernel, bn, tA, tB, out):
+    m, n, k = 300, 520, 200          # 2-3 tiles + ragged tails in m, n and k
+    _use(kernel, bn)
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), tA, tB, out=out, pad=(8, 16, 8))
+    got = case.run_gpu()
+    _expect_kernel(case, kernel)
+    c_ref, r, ab = case.oracle(oracle_mod)
+    rel = assert_within_tolerance(case, got, r, ab)
+    assert rel < 1e-5, f"precision regression: max err/absab = {rel}"
+    # padding rows of C are never written
+    assert np.all(np.isnan(case.padding(got).astype(np.float32)))
+
+
+@pytest.mark.parametrize("kernel,bn", KERNELS)
+@pytest.mark.parametrize("tA,tB", TRANS)
+@pytest.mark.parametrize("out", ["f16", "f32"])
+def test_integer_bit_exact(oracle_mod, kernel, bn, tA, tB, out):
+    m, n, k = 257, 391, 1000
+    _use(kernel, bn)
+    opA = inputs.integer_f16(m, k, 3, -4, 4)
+    opB = inputs.integer_f16(k, n, 4, -4, 4)
+    if out == "f16":  # keep |C| <= 2048 so FP16 output is exact
+        opA = (opA.astype(np.float32) / 2).round().astype(np.float16)
+    case = GpuCase(opA, opB, tA, tB, out=out)
+    got = case.run_gpu()
+    _expect_kernel(case, kernel)
+    c_ref, r, _ = case.oracle(oracle_mod)
+    if out == "f16":
+        assert np.max(np.abs(r)) <= 2048
+    assert np.array_equal(case.view(got).astype(np.float64), r)
+    assert np.array_equal(case.view(got), case.view(c_ref))
+
+
+@pytest.mark.parametrize("kernel,bn", KERNELS)
+@pytest.mark.parametrize("tA,tB", TRANS)
+def test_identity_and_permutation(oracle_mod, kernel, bn, tA, tB):
+    _use(kernel, bn)
+    k = 384
+    X = inputs.uniform_f16(k, 200, 5)
+    case = GpuCase(np.eye(k, dtype=np.float16), X, tA, tB, out="f16")
+    got = case.run_gpu()
+    assert np.array_equal(case.view(got).view(np.uint16), X.view(np.uint16))
+    perm = np.random.Generator(np.random.PCG64(8)).permutation(k)
+    P = np.eye(k, dtype=np.float16)[perm]
+    Y = inputs.uniform_f16(150, k, 6)
+    case = GpuCase(Y, P.T.copy(), tA, tB, out="f32")
+    got = case.run_gpu()
+    assert np.array_equal(case.view(got), Y[:, perm].astype(np.float32))
+
+
+@pytest.mark.parametrize("kernel,bn", KERNELS)
+@pytest.mark.parametrize("k", [4096, 8192])
+def test_accumulator_width(oracle_mod, kernel, bn, k):
+    """FP32 accumulation gets k/16 - 2 exactly; an FP16 accumulator returns 0."""
+    _use(kernel, bn)
+    a, b, expect = inputs.accumulator_width_case(256, 256, k)
+    for tA, tB in TRANS:
+        case = GpuCase(a, b, tA, tB, out="f32")
+        got = case.view(case.run_gpu())
+        assert np.all(got == expect), (tA, tB, np.unique(got)[:5])
+
+
+@pytest.mark.parametrize("kernel,bn", KERNELS)
+@pytest.mark.parametrize("alpha,beta", [(1.0, 0.0), (2.0, 1.0), (-0.5, -1.0), (1.0, 0.5), (0.25, 2.0)])
+@pytest.mark.parametrize("out", ["f16", "f32"])
+def test_alpha_beta_integer(oracle_mod, kernel, bn, alpha, beta, out):
+    _use(kernel, bn)
+    m, n, k = 200, 300, 128
+    opA = inputs.integer_f16(m, k, 9, -3, 3)
+    opB = inputs.integer_f16(k, n, 10, -3, 3)
+    C = inputs.integer_f16(m, n, 11, -64, 64)
+    case = GpuCase(opA, opB, "T", "N", alpha, beta, C=C, out=out, pad=(0, 0, 8))
+    got = case.run_gpu()
+    c_ref, r, _ = case.oracle(oracle_mod)
+    assert np.array_equal(case.view(got).astype(np.float64), r)
+
+
+@pytest.mark.parametrize("kernel,bn", KERNELS)
+@pytest.mark.parametrize("out", ["f16", "f32"])
+def test_beta_zero_never_reads_C(oracle_mod, kernel, bn, out):
+    _use(kernel, bn)
+    m, n, k = 130, 270, 96
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "N", "N", 1.0, 0.0,
+                   out=out, c_fill=np.nan)
+    got = case.view(case.run_gpu())
+    assert not np.any(np.isnan(got.astype(np.float32)))
+
+
+def test_quick_returns(oracle_mod):
+    m, n = 100, 70
+    C = inputs.uniform_f16(m, n, 3)
+    for out in ("f16", "f32"):
+        # k == 0 -> C = beta*C
+        case = GpuCase(np.zeros((m, 0), np.float16), np.zeros((0, n), np.float16), "N", "N", 1.0, 2.0,
+                       C=C, out=out)
+        got = case.view(case.run_gpu()).astype(np.float64)
+        assert np.array_equal(got, (2.0 * C.astype(np.float64)).astype(np.float16 if out == "f16" else np.float32))
+        # alpha == 0 with inf in A -> C = beta*C, A*B not evaluated
+        A = np.full((m, 5), np.inf, np.float16)
+        case = GpuCase(A, np.ones((5, n), np.float16), "N", "N", 0.0, -1.0, C=C, out=out)
+        got = case.view(case.run_gpu()).astype(np.float64)
+        assert np.array_equal(got, -C.astype(np.float64))
+        # alpha == 0, beta == 0 -> zeros without reading a NaN C
+        case = GpuCase(A, np.ones((5, n), np.float16), "N", "N", 0.0, 0.0, out=out, c_fill=np.nan)
+        got = case.view(case.run_gpu()).astype(np.float64)
+        assert np.all(got == 0)
+
+
+def test_degenerate_shapes(oracle_mod):
+    for (m, n, k) in [(1, 1, 1), (1, 300, 70), (300, 1, 70), (7, 9, 1), (129, 257, 63), (16, 16, 16)]:
+        for tA, tB in TRANS:
+            case = GpuCase(inputs.uniform_f16(m, k, m + k), inputs.uniform_f16(k, n, n + 7 * k), tA, tB, out="f32")
+            got = case.run_gpu()
+            _, r, ab = case.oracle(oracle_mod)
+            assert_within_tolerance(case, got, r, ab)
+
+
+def test_unaligned_falls_back_to_simt(oracle_mod):
+    m, n, k = 130, 70, 77
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", out="f16", pad=(3, 5, 1),
+                   align=False)
+    got = case.run_gpu()
+    assert case.stats["last_kernel"] == "simt"
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, got, r, ab)
+
+
+def test_overflow_to_inf(oracle_mod):
+    opA = np.full((128, 64), 16.0, np.float16)
+    opB = np.full((64, 128), 64.0, np.float16)      # 64 * 1024 = 65536 -> inf
+    for kernel, bn in KERNELS:
+        _use(kernel, bn)
+        case = GpuCase(opA, opB, "T", "N", out="f16")
+        got = case.view(case.run_gpu())
+        assert np.all(np.isposinf(got.astype(np.float32)))
+
+
+def test_deterministic(oracle_mod):
+    m, n, k = 1000, 700, 1500
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", out="f32")
+    a, b = case.run_gpu(repeat=2)
+    assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
+
+
+def test_all_kernels_agree_on_random(oracle_mod):
+    """Different tile shapes only change which CTA computes an element, not the K
+    order inside the tensor core, so tc1/tc2 results are bitwise identical."""
+    m, n, k = 700, 900, 640
+    base = None
+    for kernel, bn in KERNELS[:3]:
+        _use(kernel, bn)
+        case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", out="f32")
+        got = case.run_gpu()
+        if base is None:
+            base = got
+        else:
+            assert np.array_equal(got.view(np.uint32), base.view(np.uint32)), kernel
