@@ -88,7 +88,7 @@ class ClockSampler:
                 except Exception:
                     rs = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h)
                 self.samples.append((sm, mx, [k for k, v in names.items() if rs & v]))
-                time.sleep(0.05)
+                time.sleep(0.01)
         except Exception as e:  # pragma: no cover
             self.samples.append((None, None, [f"nvml-error:{type(e).__name__}"]))
 
@@ -262,18 +262,27 @@ def run_ours(args, world, rank, local):
     clocks = ClockSampler(local)
     clocks.start()
     evs = []
-    for _ in range(args.steps):
+    probe = torch.zeros(4 * args.steps, dtype=torch.int64, device=dev)   # in-kernel SM clock probe
+    for i in range(args.steps):
         flush.zero_()                                   # L2 flush, outside the events
+        binding.set_probe(probe[4 * i:])
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         step()
         e1.record(stream)
         evs.append((e0, e1))
+    binding.set_probe(None)
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
     torch.cuda.synchronize()
     clk = clocks.stop()
+    pv = probe.view(-1, 4).cpu().tolist()
+    ghz = [(c1 - c0) / (n1 - n0) for c0, n0, c1, n1 in pv if n1 > n0]
+    if ghz:
+        clk["sm_mhz_in_kernel_median"] = 1000.0 * statistics.median(ghz)
+        clk["sm_mhz_in_kernel_min"] = 1000.0 * min(ghz)
+        clk["in_kernel_how"] = "clock64 / %globaltimer deltas of CTA 0 per timed launch"
     launches = lib.hgemm_launch_count() - launches0
     step_ms = [a.elapsed_time(b) for a, b in evs]
     ms_local = statistics.mean(step_ms)
@@ -386,7 +395,7 @@ def run_ours(args, world, rank, local):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="cfg2_8192_TN_f16")

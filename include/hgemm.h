@@ -80,12 +80,13 @@ typedef enum {
     HGEMM_KERNEL_AUTO = 0,
     HGEMM_KERNEL_SIMT = 1,       /* CUDA-core fallback (always available) */
     HGEMM_KERNEL_TC_1SM = 2,     /* tcgen05 cta_group::1, tile 128 x block_n */
-    HGEMM_KERNEL_TC_2SM = 3      /* tcgen05 cta_group::2 (CTA pair), tile 256 x block_n */
+    HGEMM_KERNEL_TC_2SM = 3      /* tcgen05 cta_group::2 (CTA pair), tile 256 x block_n (256 or 512) */
 } hgemm_kernel_t;
 
 typedef struct {
     int32_t kernel;    /* hgemm_kernel_t */
-    int32_t block_n;   /* tile width along the output's contiguous dim: 64, 128 or 256 (0 = auto) */
+    int32_t block_n;   /* tile width along the output's contiguous dim: 128, 256 (1-SM, 2-SM) or
+                          512 (2-SM only); 0 = auto */
     int32_t group_m;   /* L2 raster group height in tiles (0 = auto) */
     int32_t max_ctas;  /* cap on persistent CTAs (0 = all SMs) */
 } hgemm_config_t;
@@ -103,6 +104,13 @@ hgemm_status_t hgemm_get_last_config(hgemm_config_t *out);
 
 /* Number of kernel launches hgemm() has enqueued in this process. */
 int64_t hgemm_launch_count(void);
+
+/* Diagnostic clock probe.  When `device_buf` is non-NULL (device memory of
+ * at least 4 x 8 bytes, owned by the caller), every tensor-core launch makes
+ * its CTA 0 write {clock64 at start, %globaltimer ns at start, clock64 at
+ * end, %globaltimer ns at end}; the SM clock during the kernel is
+ * (clk1-clk0)/(ns1-ns0) GHz.  NULL (the default) disables it.  Process-global. */
+hgemm_status_t hgemm_set_probe(unsigned long long *device_buf);
 
 #ifdef __cplusplus
 }

@@ -63,6 +63,8 @@ def load_library():
     lib.hgemm_set_config.restype = ctypes.c_int
     lib.hgemm_get_last_config.argtypes = [ctypes.POINTER(_Config)]
     lib.hgemm_get_last_config.restype = ctypes.c_int
+    lib.hgemm_set_probe.argtypes = [vp]
+    lib.hgemm_set_probe.restype = ctypes.c_int
     lib.hgemm_launch_count.argtypes = []
     lib.hgemm_launch_count.restype = ctypes.c_int64
     _lib = lib
@@ -86,6 +88,17 @@ def set_config(kernel: str | int = "auto", block_n: int = 0, group_m: int = 0, m
         _check(lib.hgemm_set_config(None))
     else:
         _check(lib.hgemm_set_config(ctypes.byref(_Config(kern, block_n, group_m, max_ctas))))
+
+
+def set_probe(buf=None):
+    """Enable (a >= 4-element int64 CUDA tensor) or disable (None) the kernel clock probe."""
+    _check(load_library().hgemm_set_probe(_ptr(buf) or None))
+
+
+def probe_clock_ghz(buf) -> float:
+    """SM clock of the last probed launch, from {clk0, ns0, clk1, ns1}."""
+    v = [int(x) for x in buf[:4].cpu().tolist()]
+    return (v[2] - v[0]) / max(v[3] - v[1], 1)
 
 
 def get_stats() -> dict:

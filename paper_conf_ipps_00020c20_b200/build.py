@@ -33,20 +33,26 @@ def needs_build() -> bool:
     return any(os.path.getmtime(s) > t for s in sources())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
+    """Compile csrc/hgemm_api.cu into `out` (default: the in-tree libhgemm.so).
+    `defines` adds -D flags (experiment variants are built to other paths)."""
+    target = out or LIB
+    if not force and out is None and not defines and not needs_build():
         return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = target + f".tmp{os.getpid()}"
     watchdog = os.environ.get("HGEMM_WATCHDOG_CYCLES", "4000000000")
     cmd = [NVCC, *ARCH, f"-DHGEMM_WATCHDOG_CYCLES={watchdog}ll", "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-shared",
            "-I", os.path.join(ROOT, "include"), "-o", tmp, os.path.join(CSRC, "hgemm_api.cu")]
+    cmd[1:1] = [f"-D{d}" for d in defines]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose="--verbose" in sys.argv)
-    print(LIB)
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv, defines=defs,
+                out=outs[0] if outs else None))

@@ -40,6 +40,7 @@ std::mutex g_mu;
 hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0};
 hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0};
 std::atomic<int64_t> g_launches{0};
+std::atomic<unsigned long long *> g_probe{nullptr};
 
 bool device_info(int dev, DeviceInfo &out) {
   if (dev < 0 || dev >= kMaxDevices) return false;
@@ -80,26 +81,29 @@ EncodeTiledFn encode_fn() {
   return fn;
 }
 
-// 2-D FP16 tensor: `inner` contiguous elements per line, `outer` lines `ld` elements apart.
+// 2-D tensor with 128-B swizzled boxes: `inner` contiguous elements per line,
+// `outer` lines `ld` elements apart.  FP16 operands (loads) or the FP16/FP32
+// output D (epilogue stores).
 bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer, int64_t ld, uint32_t box_inner,
-              uint32_t box_outer) {
+              uint32_t box_outer, bool f32 = false) {
   EncodeTiledFn fn = encode_fn();
   if (!fn) return false;
+  const int esz = f32 ? 4 : 2;
   cuuint64_t dims[2] = {inner, outer};
-  cuuint64_t strides[1] = {static_cast<cuuint64_t>(ld) * 2};
+  cuuint64_t strides[1] = {static_cast<cuuint64_t>(ld) * esz};
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t estr[2] = {1, 1};
-  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(base), dims, strides, box, estr,
-                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  CUresult r = fn(map, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2,
+                  const_cast<void *>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS;
 }
 
 // ----------------------------------------------------------------- TC launch
 template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32>
-hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const TcParams &p, int dev,
-                         const DeviceInfo &di, int max_ctas, cudaStream_t stream) {
-  using S = TcShape<BN, CG>;
+hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &td, const TcParams &p,
+                         int dev, const DeviceInfo &di, int max_ctas, cudaStream_t stream) {
+  using S = TcShape<BN, CG, OUT_F32>;
   auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32>;
   static int attr_done[kMaxDevices] = {};
   static int max_clusters[kMaxDevices] = {};
@@ -142,17 +146,18 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const TcP
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (cudaLaunchKernelEx(&cfg, kern, ta, tb, p) != cudaSuccess) return HGEMM_ERR_CUDA;
+  if (cudaLaunchKernelEx(&cfg, kern, ta, tb, td, p) != cudaSuccess) return HGEMM_ERR_CUDA;
   g_launches.fetch_add(1, std::memory_order_relaxed);
   return HGEMM_SUCCESS;
 }
 
 template <int BN, int CG>
 hgemm_status_t dispatch_tc_layout(bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
-                                  const TcParams &p, int dev, const DeviceInfo &di, int max_ctas, cudaStream_t s) {
+                                  const CUtensorMap &td, const TcParams &p, int dev, const DeviceInfo &di,
+                                  int max_ctas, cudaStream_t s) {
 #define HG_CASE(AM, BM_, F)                                                               \
   if (a_mn == AM && b_mn == BM_ && f32 == F)                                              \
-    return launch_tc<BN, CG, AM, BM_, F>(ta, tb, p, dev, di, max_ctas, s);
+    return launch_tc<BN, CG, AM, BM_, F>(ta, tb, td, p, dev, di, max_ctas, s);
   HG_CASE(false, false, false)
   HG_CASE(false, false, true)
   HG_CASE(false, true, false)
@@ -171,13 +176,15 @@ inline bool is_n(char c) { return c == 'N' || c == 'n'; }
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 // Automatic tile choice: estimated time = waves * per-wave tile cost.
-void choose_tc(int64_t M, int64_t N, int num_sms, int &cg, int &bn) {
+void choose_tc(int64_t M, int64_t N, int num_sms, int forced_cg, int &cg, int &bn) {
   struct Cand { int cg, bn; double eff; };
-  // eff: relative per-SM throughput of the tile shape (2-SM 256x256 halves
-  // the L2->SM operand traffic per FLOP; 128x128 needs 1.5x the bytes/FLOP of 128x256).
-  const Cand cands[3] = {{2, 256, 1.00}, {1, 256, 0.93}, {1, 128, 0.80}};
+  // eff: relative per-SM throughput of the tile shape.  Larger tiles move
+  // fewer L2->SMEM bytes per FLOP (pair 256x512: 171 FLOP/B, 256x256: 128,
+  // 1-SM 128x256: 85, 128x128: 64), which under the 1 kW power cap buys clock.
+  const Cand cands[4] = {{2, 512, 1.00}, {2, 256, 0.93}, {1, 256, 0.85}, {1, 128, 0.75}};
   double best = 1e300;
   for (const Cand &c : cands) {
+    if (forced_cg && c.cg != forced_cg) continue;
     const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, c.bn);
     const int64_t units = num_sms / c.cg;
     const int64_t waves = cdiv(tiles, units);
@@ -207,8 +214,10 @@ hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
     return HGEMM_SUCCESS;
   }
   if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_TC_2SM) return HGEMM_ERR_INVALID_VALUE;
-  if (cfg->block_n != 0 && cfg->block_n != 128 && cfg->block_n != 256) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->block_n != 0 && cfg->block_n != 128 && cfg->block_n != 256 && cfg->block_n != 512)
+    return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_TC_2SM && cfg->block_n == 128) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->kernel == HGEMM_KERNEL_TC_1SM && cfg->block_n == 512) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->group_m < 0 || cfg->max_ctas < 0) return HGEMM_ERR_INVALID_VALUE;
   g_cfg = *cfg;
   return HGEMM_SUCCESS;
@@ -222,6 +231,11 @@ hgemm_status_t hgemm_get_last_config(hgemm_config_t *out) {
 }
 
 int64_t hgemm_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
+
+hgemm_status_t hgemm_set_probe(unsigned long long *device_buf) {
+  g_probe.store(device_buf, std::memory_order_relaxed);
+  return HGEMM_SUCCESS;
+}
 
 hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A, int64_t lda, const void *B,
                      int64_t ldb, float beta, void *C, int64_t ldc, char transA, char transB,
@@ -291,11 +305,11 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
 
   // ---------------------------------------------------------- tcgen05 path
   const int64_t M = n, N = m;  // kernel coordinates (D = C^T)
-  int cg = 2, bn = 256;
-  if (cfg.kernel == HGEMM_KERNEL_TC_1SM) { cg = 1; bn = cfg.block_n ? cfg.block_n : 256; }
-  else if (cfg.kernel == HGEMM_KERNEL_TC_2SM) { cg = 2; bn = 256; }
-  else choose_tc(M, N, di.num_sms, cg, bn);
-  const int bn_cta = bn / cg;
+  int cg = 2, bn = 512;
+  const int forced_cg = cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
+  if (forced_cg && cfg.block_n) { cg = forced_cg; bn = cfg.block_n; }
+  else choose_tc(M, N, di.num_sms, forced_cg, cg, bn);
+  const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
 
   const bool a_mn = tB;   // Ak = op(B)^T: 'T' -> rows of Ak contiguous along M
   const bool b_mn = !tA;  // Bk = op(A):   'N' -> rows of Bk contiguous along N
@@ -304,9 +318,12 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
   else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
   if (ok) {
-    if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, bn_cta);
+    if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, b_rows);
     else ok = make_map(&tb, A, static_cast<uint64_t>(m), static_cast<uint64_t>(k), lda, 64, 64);
   }
+  // D = C^T row-major (N = m contiguous), stored in 32-row x 128-B swizzled boxes
+  CUtensorMap td;
+  if (ok) ok = make_map(&td, C, static_cast<uint64_t>(m), static_cast<uint64_t>(n), ldc, f32 ? 32 : 64, 32, f32);
   if (!ok) return HGEMM_ERR_CUDA;
 
   TcParams p;
@@ -318,15 +335,25 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
   p.group_m = cfg.group_m > 0 ? cfg.group_m : 8;
   p.group_m = std::max(1, std::min(p.group_m, p.num_m_tiles));
+  {
+    const char *e = std::getenv("HGEMM_L2_HINT");
+    p.l2_hint = e ? std::atoi(e) : 0;
+  }
+  p.probe = g_probe.load(std::memory_order_relaxed);
   p.alpha = alpha;
   p.beta = beta;
   p.D = C;
   p.ldd = ldc;
 
   hgemm_status_t st;
-  if (cg == 2) st = dispatch_tc_layout<256, 2>(a_mn, b_mn, f32, ta, tb, p, dev, di, cfg.max_ctas, stream);
-  else if (bn == 256) st = dispatch_tc_layout<256, 1>(a_mn, b_mn, f32, ta, tb, p, dev, di, cfg.max_ctas, stream);
-  else st = dispatch_tc_layout<128, 1>(a_mn, b_mn, f32, ta, tb, p, dev, di, cfg.max_ctas, stream);
+  if (cg == 2 && bn == 512)
+    st = dispatch_tc_layout<512, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
+  else if (cg == 2)
+    st = dispatch_tc_layout<256, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
+  else if (bn == 256)
+    st = dispatch_tc_layout<256, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
+  else
+    st = dispatch_tc_layout<128, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);
     g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas};

@@ -1,6 +1,6 @@
 // Persistent, warp-specialised tcgen05 HGEMM for sm_100a.
 //
-// Kernel coordinates.  The kernel computes a ROW-MAJOR tile matrix
+// Kernel coordinates.  The kernel computes a ROW-MAJOR matrix
 //     D[M x N] = alpha * Ak[M x K] * Bk[N x K]^T + beta * D,      D[r][c] at D + r*ldd + c
 // where Ak feeds the UMMA "A" operand (rows -> TMEM lanes) and Bk the UMMA
 // "B" operand (rows -> TMEM columns).  The host maps the column-major ABI
@@ -9,8 +9,12 @@
 // writes contiguous runs of m.
 //
 // Paper mapping:
-//   Alg. 1 P:248-272 two-level blocking      -> CTA tile 128 x BN (x2 for the CTA pair),
-//                                               k-block BK = 64 (one 128-B swizzle atom)
+//   Alg. 1 P:248-272 two-level blocking      -> cluster tile (128*CG) x BN, k-block BK = 64
+//                                               (one 128-B swizzle atom); the paper's
+//                                               256x256 CTA block (Table VII) becomes a
+//                                               256x512 CTA-pair tile (128 FLOP/B -> 171 FLOP/B
+//                                               of L2->SMEM traffic, the SVI-A.2 intensity
+//                                               argument b_m*b_n/(b_m+b_n) of P:276)
 //   SVI-A.2 P:274 grid of ceil(m/bm) x ceil(n/bn) blocks
 //                                             -> persistent clusters walking an
 //                                               L2-grouped raster (future work at P:460)
@@ -24,9 +28,13 @@
 //   warp 0     : TMA producer (one elected lane)
 //   warp 1     : TMEM allocator; in the leader CTA, the MMA issuer (one lane)
 //   warps 2..5 : epilogue, TMEM lanes 32*(warp%4) .. +31
-// Pipelines: smem ring full[s]/empty[s]; accumulator double buffer
-// tmem_full[2]/tmem_empty[2] so the epilogue of tile i overlaps the
-// mainloop of tile i+1.
+// Pipelines: smem ring full[s]/empty[s]; accumulator hand-off tmem_full[buf] /
+// tmem_empty[buf][half].  BN <= 256 double-buffers the accumulator (epilogue of
+// tile i overlaps the mainloop of tile i+1).  BN = 512 fills TMEM (512 columns)
+// with one accumulator split in two 256-column halves that are released
+// separately, so the next tile's first half of MMAs overlaps the drain of the
+// second half.  The epilogue stages 32 x 128-B boxes in swizzled shared memory
+// and writes them with TMA bulk stores.
 #pragma once
 #include <cuda_fp16.h>
 
@@ -35,13 +43,15 @@
 namespace hg {
 
 struct TcParams {
-  int32_t M, N, K;                 // D is M x N, reduction length K
+  int32_t M, N, K;                   // D is M x N, reduction length K
   int32_t num_m_tiles, num_n_tiles;  // in cluster tiles (128*CG x BN)
   int32_t num_k_blocks;
-  int32_t group_m;                 // raster group height, in m-tiles
+  int32_t group_m;                   // raster group height, in m-tiles
+  int32_t l2_hint;                   // 0: evict_normal for both; 1: Ak evict_last, Bk evict_first
   float alpha, beta;
   void *D;
   int64_t ldd;
+  unsigned long long *probe;         // diagnostic (may be null): CTA 0 writes {clk0, ns0, clk1, ns1}
 };
 
 // UMMA shared-memory descriptor, SWIZZLE_128B, K-major operand.
@@ -95,109 +105,49 @@ __device__ __forceinline__ uint32_t pack_half2(float a, float b) {
   return *reinterpret_cast<uint32_t *>(&h);
 }
 
-// Epilogue for one thread: 32 consecutive columns [col, col+32) of row `row`.
-template <bool OUT_F32>
-__device__ __forceinline__ void store_chunk(const TcParams &p, int row, int col, const uint32_t (&v)[32]) {
-  if (row >= p.M || col >= p.N) return;
-  const int ncol = min(32, p.N - col);
-  const float alpha = p.alpha, beta = p.beta;
-  if constexpr (OUT_F32) {
-    float *dst = static_cast<float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
-    if (ncol == 32) {
-      float4 *d4 = reinterpret_cast<float4 *>(dst);
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        float4 o;
-        o.x = alpha * __uint_as_float(v[4 * q + 0]);
-        o.y = alpha * __uint_as_float(v[4 * q + 1]);
-        o.z = alpha * __uint_as_float(v[4 * q + 2]);
-        o.w = alpha * __uint_as_float(v[4 * q + 3]);
-        if (beta != 0.0f) {
-          const float4 c = d4[q];
-          o.x = fmaf(beta, c.x, o.x);
-          o.y = fmaf(beta, c.y, o.y);
-          o.z = fmaf(beta, c.z, o.z);
-          o.w = fmaf(beta, c.w, o.w);
-        }
-        d4[q] = o;
-      }
-    } else {
-#pragma unroll
-      for (int j = 0; j < 32; ++j) {
-        if (j < ncol) {
-          float o = alpha * __uint_as_float(v[j]);
-          if (beta != 0.0f) o = fmaf(beta, dst[j], o);
-          dst[j] = o;
-        }
-      }
-    }
-  } else {
-    __half *dst = static_cast<__half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
-    if (ncol == 32) {
-      uint4 *d4 = reinterpret_cast<uint4 *>(dst);
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        float f[8];
-#pragma unroll
-        for (int e = 0; e < 8; ++e) f[e] = alpha * __uint_as_float(v[8 * q + e]);
-        if (beta != 0.0f) {
-          const uint4 c = d4[q];
-          const __half2 *ch = reinterpret_cast<const __half2 *>(&c);
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const float2 cf = __half22float2(ch[e]);
-            f[2 * e] = fmaf(beta, cf.x, f[2 * e]);
-            f[2 * e + 1] = fmaf(beta, cf.y, f[2 * e + 1]);
-          }
-        }
-        uint4 o;
-        o.x = pack_half2(f[0], f[1]);
-        o.y = pack_half2(f[2], f[3]);
-        o.z = pack_half2(f[4], f[5]);
-        o.w = pack_half2(f[6], f[7]);
-        d4[q] = o;
-      }
-    } else {
-#pragma unroll
-      for (int j = 0; j < 32; ++j) {
-        if (j < ncol) {
-          float o = alpha * __uint_as_float(v[j]);
-          if (beta != 0.0f) o = fmaf(beta, __half2float(dst[j]), o);
-          dst[j] = __float2half_rn(o);
-        }
-      }
-    }
-  }
-}
-
-template <int BN, int CG>
+template <int BN, int CG, bool OUT_F32>
 struct TcShape {
-  static constexpr int BM = 128;  // rows per CTA (TMEM lanes)
-  static constexpr int BK = 64;   // FP16 per 128-B swizzle atom
-  static constexpr int BN_CTA = BN / CG;
+  static constexpr int BM = 128;                       // rows per CTA (TMEM lanes)
+  static constexpr int BK = 64;                        // FP16 per 128-B swizzle atom
+  static constexpr int UMMA_N = BN > 256 ? 256 : BN;   // N of one tcgen05.mma
+  static constexpr int NH = BN / UMMA_N;               // accumulator halves per tile
+  static constexpr int B_ROWS = UMMA_N / CG;           // Bk rows per CTA per half
   static constexpr uint32_t A_BYTES = BM * BK * 2;
-  static constexpr uint32_t B_BYTES = BN_CTA * BK * 2;
+  static constexpr uint32_t B_HALF_BYTES = B_ROWS * BK * 2;
+  static constexpr uint32_t B_BYTES = NH * B_HALF_BYTES;
   static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (STAGE_BYTES <= 32768) ? 6 : 4;
-  static constexpr uint32_t TMEM_COLS = (2 * BN <= 64) ? 64 : (2 * BN <= 128) ? 128 : (2 * BN <= 256) ? 256 : 512;
-  static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*barriers*/ + 1024 /*alignment*/;
-  static_assert(BN % 32 == 0 && BN >= 64 && BN <= 256, "BN");
-  static_assert(BN_CTA % 64 == 0, "BN_CTA");
+  static constexpr int ACC = (2 * BN <= 512) ? 2 : 1;  // accumulator buffers in TMEM
+  static constexpr uint32_t TMEM_COLS = (ACC * BN <= 256) ? 256 : 512;
+  static constexpr int EPI_COLS = OUT_F32 ? 32 : 64;   // one 128-B staging row per thread
+  static constexpr uint32_t EPI_BYTES = 4 * 2 * 32 * 128;  // 4 warps x 2 buffers x 32 rows x 128 B
+  // As many ring stages as fit in 227 KB next to the staging buffers, barriers and alignment slack.
+  static constexpr int STAGES_FIT = static_cast<int>((227u * 1024u - EPI_BYTES - 2048u) / STAGE_BYTES);
+  static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
+  static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + EPI_BYTES + 1024 /*barriers*/ + 1024 /*align*/;
+  static_assert(BN % 64 == 0 && BN >= 128 && BN <= 512, "BN");
+  static_assert(B_ROWS % 64 == 0, "B_ROWS");
+  static_assert(STAGES >= 3, "stages");
+  static_assert(UMMA_N % EPI_COLS == 0, "epilogue chunking");
 };
 
 template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32>
 __global__ void __launch_bounds__(192, 1)
     hgemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                    const TcParams p) {
+                    const __grid_constant__ CUtensorMap tmD, const TcParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
-  using S = TcShape<BN, CG>;
+  using S = TcShape<BN, CG, OUT_F32>;
   constexpr int BM = S::BM;
   constexpr int BK = S::BK;
-  constexpr int BN_CTA = S::BN_CTA;
+  constexpr int UMMA_N = S::UMMA_N;
+  constexpr int NH = S::NH;
+  constexpr int B_ROWS = S::B_ROWS;
   constexpr int STAGES = S::STAGES;
+  constexpr int ACC = S::ACC;
+  constexpr int EPI_COLS = S::EPI_COLS;
   constexpr uint32_t A_BYTES = S::A_BYTES;
+  constexpr uint32_t B_HALF_BYTES = S::B_HALF_BYTES;
   constexpr uint32_t STAGE_BYTES = S::STAGE_BYTES;
-  constexpr uint32_t IDESC = make_idesc_f16<BM * CG, BN, A_MN, B_MN>();
+  constexpr uint32_t IDESC = make_idesc_f16<BM * CG, UMMA_N, A_MN, B_MN>();
   // Per-K=16 advance of the descriptor start address (in bytes).
   constexpr uint32_t A_KSTEP = A_MN ? 16 * 128 : 32;
   constexpr uint32_t B_KSTEP = B_MN ? 16 * 128 : 32;
@@ -205,11 +155,12 @@ __global__ void __launch_bounds__(192, 1)
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw_u32 = smem_u32(smem_raw);
   uint8_t *smem = smem_raw + ((1024u - (raw_u32 & 1023u)) & 1023u);
-  uint64_t *full = reinterpret_cast<uint64_t *>(smem + STAGES * STAGE_BYTES);
+  uint8_t *epi_smem = smem + STAGES * STAGE_BYTES;
+  uint64_t *full = reinterpret_cast<uint64_t *>(epi_smem + S::EPI_BYTES);
   uint64_t *empty = full + STAGES;
-  uint64_t *tfull = empty + STAGES;
-  uint64_t *tempty = tfull + 2;
-  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + 2);
+  uint64_t *tfull = empty + STAGES;      // [ACC]
+  uint64_t *tempty = tfull + ACC;        // [ACC][NH]
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + ACC * NH);
 
   const uint32_t warp = warp_id();
   const uint32_t lane = lane_id();
@@ -221,6 +172,7 @@ __global__ void __launch_bounds__(192, 1)
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
+    tma_prefetch_desc(&tmD);
   }
   if (warp == 1) {
     if (lane == 0) {
@@ -228,9 +180,9 @@ __global__ void __launch_bounds__(192, 1)
         mbar_init(&full[s], 1);
         mbar_init(&empty[s], 1);
       }
-      for (int a = 0; a < 2; ++a) {
+      for (int a = 0; a < ACC; ++a) {
         mbar_init(&tfull[a], 1);
-        mbar_init(&tempty[a], 4 * CG);
+        for (int h = 0; h < NH; ++h) mbar_init(&tempty[a * NH + h], 4 * CG);
       }
       fence_mbarrier_init();
     }
@@ -241,17 +193,25 @@ __global__ void __launch_bounds__(192, 1)
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  unsigned long long probe_clk = 0, probe_ns = 0;
+  if (p.probe != nullptr && blockIdx.x == 0 && threadIdx.x == 0) {
+    probe_clk = clock64();
+    probe_ns = globaltimer_ns();
+  }
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer
     if (lane == 0) {
-      const uint64_t pol = l2_policy_evict_normal();
+      // Raster groups sweep N with group_m M-tiles held: the Ak panels are
+      // re-read by the next waves of the group, the Bk panels only within a wave.
+      const uint64_t pol_a = p.l2_hint == 1 ? l2_policy_evict_last() : l2_policy_evict_normal();
+      const uint64_t pol_b = p.l2_hint == 1 ? l2_policy_evict_first() : l2_policy_evict_normal();
       uint32_t stage = 0, phase = 0;
       for (int t = cluster_id; t < num_tiles; t += num_clusters) {
         int tm, tn;
         tile_coords(t, p, tm, tn);
         const int a_row = tm * BM * CG + static_cast<int>(rank) * BM;
-        const int b_row = tn * BN + static_cast<int>(rank) * BN_CTA;
+        const int b_row0 = tn * BN + static_cast<int>(rank) * B_ROWS;
         for (int kb = 0; kb < p.num_k_blocks; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1u);
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
@@ -266,23 +226,28 @@ __global__ void __launch_bounds__(192, 1)
           }
           const int k0 = kb * BK;
           if constexpr (!A_MN) {
-            if constexpr (CG == 1) tma_load_2d(&tmA, sa, fb, k0, a_row, pol);
-            else tma_load_2d_pair(&tmA, sa, fb, k0, a_row, pol);
+            if constexpr (CG == 1) tma_load_2d(&tmA, sa, fb, k0, a_row, pol_a);
+            else tma_load_2d_pair(&tmA, sa, fb, k0, a_row, pol_a);
           } else {
 #pragma unroll
-            for (int h = 0; h < BM / 64; ++h) {
-              if constexpr (CG == 1) tma_load_2d(&tmA, sa + h * 8192, fb, a_row + 64 * h, k0, pol);
-              else tma_load_2d_pair(&tmA, sa + h * 8192, fb, a_row + 64 * h, k0, pol);
+            for (int q = 0; q < BM / 64; ++q) {
+              if constexpr (CG == 1) tma_load_2d(&tmA, sa + q * 8192, fb, a_row + 64 * q, k0, pol_a);
+              else tma_load_2d_pair(&tmA, sa + q * 8192, fb, a_row + 64 * q, k0, pol_a);
             }
           }
-          if constexpr (!B_MN) {
-            if constexpr (CG == 1) tma_load_2d(&tmB, sb, fb, k0, b_row, pol);
-            else tma_load_2d_pair(&tmB, sb, fb, k0, b_row, pol);
-          } else {
 #pragma unroll
-            for (int h = 0; h < BN_CTA / 64; ++h) {
-              if constexpr (CG == 1) tma_load_2d(&tmB, sb + h * 8192, fb, b_row + 64 * h, k0, pol);
-              else tma_load_2d_pair(&tmB, sb + h * 8192, fb, b_row + 64 * h, k0, pol);
+          for (int h = 0; h < NH; ++h) {
+            const uint32_t sbh = sb + h * B_HALF_BYTES;
+            const int b_row = b_row0 + h * UMMA_N;
+            if constexpr (!B_MN) {
+              if constexpr (CG == 1) tma_load_2d(&tmB, sbh, fb, k0, b_row, pol_b);
+              else tma_load_2d_pair(&tmB, sbh, fb, k0, b_row, pol_b);
+            } else {
+#pragma unroll
+              for (int q = 0; q < B_ROWS / 64; ++q) {
+                if constexpr (CG == 1) tma_load_2d(&tmB, sbh + q * 8192, fb, b_row + 64 * q, k0, pol_b);
+                else tma_load_2d_pair(&tmB, sbh + q * 8192, fb, b_row + 64 * q, k0, pol_b);
+              }
             }
           }
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
@@ -295,65 +260,182 @@ __global__ void __launch_bounds__(192, 1)
       uint32_t stage = 0, phase = 0;
       int it = 0;
       for (int t = cluster_id; t < num_tiles; t += num_clusters, ++it) {
-        const uint32_t acc = it & 1;
-        const uint32_t acc_phase = (it >> 1) & 1;
-        if constexpr (CG == 2) mbar_wait_cluster(&tempty[acc], acc_phase ^ 1u);
-        else mbar_wait(&tempty[acc], acc_phase ^ 1u);
-        tc_fence_after();
-        const uint32_t d_tmem = tmem_base + acc * BN;
+        const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
+        const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
+        const uint32_t d_tmem = tmem_base + buf * BN;
         for (int kb = 0; kb < p.num_k_blocks; ++kb) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
           const uint32_t sb = sa + A_BYTES;
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k) {
-            const uint64_t ad = A_MN ? sdesc_mn_sw128(sa + k * A_KSTEP, 8192) : sdesc_k_sw128(sa + k * A_KSTEP);
-            const uint64_t bd = B_MN ? sdesc_mn_sw128(sb + k * B_KSTEP, 8192) : sdesc_k_sw128(sb + k * B_KSTEP);
-            umma_f16<CG>(d_tmem, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
+          for (int h = 0; h < NH; ++h) {
+            if (kb == 0) {
+              // this accumulator half must have been drained by the previous tile's epilogue
+              if constexpr (CG == 2) mbar_wait_cluster(&tempty[buf * NH + h], acc_phase ^ 1u);
+              else mbar_wait(&tempty[buf * NH + h], acc_phase ^ 1u);
+              tc_fence_after();
+            }
+#pragma unroll
+            for (int k = 0; k < BK / 16; ++k) {
+              const uint32_t a_addr = sa + k * A_KSTEP;
+              const uint32_t b_addr = sb + h * B_HALF_BYTES + k * B_KSTEP;
+              const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+              const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
+              umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
+            }
           }
           umma_commit<CG>(&empty[stage]);  // frees the smem stage once these MMAs retire
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
         }
-        umma_commit<CG>(&tfull[acc]);      // accumulator ready for the epilogue
+        umma_commit<CG>(&tfull[buf]);      // accumulator ready for the epilogue
       }
     }
   } else {
     // ------------------------------------------------------------ epilogue warps
     const uint32_t quad = warp & 3u;
+    const uint32_t stg = smem_u32(epi_smem) + quad * (2u * 32u * 128u);  // this warp's 2 x 4 KB staging
     const uint32_t tempty_addr = (CG == 2) ? mapa_shared(smem_u32(&tempty[0]), 0) : smem_u32(&tempty[0]);
+    const float alpha = p.alpha, beta = p.beta;
+    uint32_t nstore = 0;
     int it = 0;
     for (int t = cluster_id; t < num_tiles; t += num_clusters, ++it) {
       int tm, tn;
       tile_coords(t, p, tm, tn);
-      const uint32_t acc = it & 1;
-      const uint32_t acc_phase = (it >> 1) & 1;
-      mbar_wait(&tfull[acc], acc_phase);
+      const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
+      const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
+      mbar_wait_sleep(&tfull[buf], acc_phase);
       tc_fence_after();
-      const int row = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad * 32 + lane);
-      const int col0 = tn * BN;
-      const uint32_t tbase = tmem_base + ((quad * 32u) << 16) + acc * BN;
+      const int row_base = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad) * 32;
+      const int row = row_base + static_cast<int>(lane);
+      const uint32_t tbase = tmem_base + ((quad * 32u) << 16) + buf * BN;
 #pragma unroll 1
-      for (int c = 0; c < BN / 32; ++c) {
-        uint32_t v[32];
-        tmem_ld_32x32b_x32(tbase + c * 32, v);
-        tmem_ld_wait();
-        if (c == BN / 32 - 1) {
-          // All TMEM reads of this accumulator are done: hand it back to the MMA warp.
-          tc_fence_before();
+      for (int h = 0; h < NH; ++h) {
+#pragma unroll 1
+        for (int c = 0; c < UMMA_N / EPI_COLS; ++c) {
+          const int colt = h * UMMA_N + c * EPI_COLS;  // column within the tile (= TMEM column offset)
+          uint32_t v[64];
+          tmem_ld_32x32b_x32(tbase + colt, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+          if constexpr (EPI_COLS == 64) tmem_ld_32x32b_x32(tbase + colt + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+          tmem_ld_wait();
+          if (c == UMMA_N / EPI_COLS - 1) {
+            // every TMEM read of this half is done: hand it back to the MMA warp
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) {
+              if constexpr (CG == 2) mbar_arrive_cluster(tempty_addr + (buf * NH + h) * 8);
+              else mbar_arrive(&tempty[buf * NH + h]);
+            }
+          }
+          // alpha*acc (+ beta*C) in FP32, packed into 32 words = one 128-B row
+          uint32_t w[32];
+          const int col = tn * BN + colt;
+          if constexpr (OUT_F32) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) w[j] = __float_as_uint(alpha * __uint_as_float(v[j]));
+          } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+              w[j] = pack_half2(alpha * __uint_as_float(v[2 * j]), alpha * __uint_as_float(v[2 * j + 1]));
+          }
+          if (beta != 0.0f && row < p.M) {
+            const int ncol = min(EPI_COLS, p.N - col);
+            if constexpr (OUT_F32) {
+              const float *src = static_cast<const float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+              if (ncol == 32) {
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                  const float4 cv = reinterpret_cast<const float4 *>(src)[q];
+                  w[4 * q + 0] = __float_as_uint(fmaf(beta, cv.x, alpha * __uint_as_float(v[4 * q + 0])));
+                  w[4 * q + 1] = __float_as_uint(fmaf(beta, cv.y, alpha * __uint_as_float(v[4 * q + 1])));
+                  w[4 * q + 2] = __float_as_uint(fmaf(beta, cv.z, alpha * __uint_as_float(v[4 * q + 2])));
+                  w[4 * q + 3] = __float_as_uint(fmaf(beta, cv.w, alpha * __uint_as_float(v[4 * q + 3])));
+                }
+              } else {
+#pragma unroll
+                for (int j = 0; j < 32; ++j)
+                  if (j < ncol) w[j] = __float_as_uint(fmaf(beta, src[j], alpha * __uint_as_float(v[j])));
+              }
+            } else {
+              const __half *src = static_cast<const __half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+              if (ncol == 64) {
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                  const uint4 cv = reinterpret_cast<const uint4 *>(src)[q];
+                  const uint32_t cw[4] = {cv.x, cv.y, cv.z, cv.w};
+#pragma unroll
+                  for (int e = 0; e < 4; ++e) {
+                    const float2 cf = __half22float2(*reinterpret_cast<const __half2 *>(&cw[e]));
+                    const int j = 4 * q + e;
+                    w[j] = pack_half2(fmaf(beta, cf.x, alpha * __uint_as_float(v[2 * j])),
+                                      fmaf(beta, cf.y, alpha * __uint_as_float(v[2 * j + 1])));
+                  }
+                }
+              } else {
+#pragma unroll
+                for (int j = 0; j < 32; ++j) {
+                  const float c0 = (2 * j < ncol) ? __half2float(src[2 * j]) : 0.0f;
+                  const float c1 = (2 * j + 1 < ncol) ? __half2float(src[2 * j + 1]) : 0.0f;
+                  w[j] = pack_half2(fmaf(beta, c0, alpha * __uint_as_float(v[2 * j])),
+                                    fmaf(beta, c1, alpha * __uint_as_float(v[2 * j + 1])));
+                }
+              }
+            }
+          }
+          // TMA bounds-checks stores at 16-B granularity along the contiguous
+          // dimension: a chunk that crosses an N that is not a multiple of 16 B
+          // (possible only in the last column tile) is written with plain stores.
+          constexpr int VEC = OUT_F32 ? 4 : 8;
+          if ((p.N & (VEC - 1)) != 0 && col + EPI_COLS > p.N) {
+            if (row < p.M) {
+              if constexpr (OUT_F32) {
+                float *dst = static_cast<float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+#pragma unroll
+                for (int j = 0; j < 32; ++j)
+                  if (col + j < p.N) dst[j] = __uint_as_float(w[j]);
+              } else {
+                __half *dst = static_cast<__half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+#pragma unroll
+                for (int j = 0; j < 32; ++j) {
+                  const __half2 hv = *reinterpret_cast<const __half2 *>(&w[j]);
+                  if (col + 2 * j < p.N) dst[2 * j] = __low2half(hv);
+                  if (col + 2 * j + 1 < p.N) dst[2 * j + 1] = __high2half(hv);
+                }
+              }
+            }
+            continue;
+          }
+          // stage the 32 x 128-B box (SWIZZLE_128B: 16-B chunk q of row r at q ^ (r % 8))
+          const uint32_t sbuf = stg + (nstore & 1u) * (32u * 128u);
+          if (nstore >= 2) {
+            if (lane == 0) bulk_wait_group_read<1>();  // the store that used this buffer has read it
+            __syncwarp();
+          }
+          const uint32_t rowaddr = sbuf + lane * 128u;
+#pragma unroll
+          for (int q = 0; q < 8; ++q)
+            st_shared_v4(rowaddr + ((q ^ (lane & 7u)) << 4), w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
+          fence_proxy_async_smem();
           __syncwarp();
           if (lane == 0) {
-            if constexpr (CG == 2) mbar_arrive_cluster(tempty_addr + acc * 8);
-            else mbar_arrive(&tempty[acc]);
+            tma_store_2d(&tmD, sbuf, col, row_base);  // the TMA unit clips rows >= M
+            bulk_commit_group();
           }
+          ++nstore;
         }
-        store_chunk<OUT_F32>(p, row, col0 + c * 32, v);
       }
     }
+    if (lane == 0) bulk_wait_group<0>();
   }
 
   tc_fence_before();
   __syncthreads();
+  if (p.probe != nullptr && blockIdx.x == 0 && threadIdx.x == 0) {
+    p.probe[0] = probe_clk;
+    p.probe[1] = probe_ns;
+    p.probe[2] = clock64();
+    p.probe[3] = globaltimer_ns();
+  }
   if constexpr (CG == 2) cluster_sync();
   if (warp == 1) {
     tc_fence_after();

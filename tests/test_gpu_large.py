@@ -62,8 +62,9 @@ def _check_sampled(oracle_mod, m, n, k, tA, tB, alpha, beta, out, seed=100):
     bound = tolerance(r, ab, alpha, beta, cvals, out, g)
     bad = ~(np.abs(g - r) <= bound)
     assert not bad.any(), f"{bad.sum()} sampled entries out of tolerance"
-    rel = float(np.max(np.abs(g - r) / np.maximum(ab, 1e-30)))
-    assert rel < 1e-5, rel
+    if out == "f32":
+        rel = float(np.max(np.abs(g - r) / np.maximum(ab, 1e-30)))
+        assert rel < 1e-5, rel
     return got, binding.get_stats()
 
 
@@ -112,7 +113,7 @@ def test_hgemm_torch_layouts(oracle_mod):
         for Bop in (B, B.t().contiguous().t()):
             C = hgemm_torch(Aop, Bop, out_dtype=torch.float32)
             assert np.all(np.abs(C.cpu().numpy() - exact) <= 1e-3 * absab)
-    C0 = torch.from_numpy(inputs.uniform_f16(M, N, 3)).cuda()
+    C0 = torch.from_numpy(np.ascontiguousarray(inputs.uniform_f16(M, N, 3))).cuda()
     C = C0.clone()
     hgemm_torch(A, B, C, alpha=0.5, beta=2.0)
     want = 0.5 * exact + 2.0 * C0.double().cpu().numpy()
