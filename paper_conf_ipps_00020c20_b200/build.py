@@ -40,7 +40,9 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     if not force and out is None and not defines and not needs_build():
         return LIB
     tmp = target + f".tmp{os.getpid()}"
-    watchdog = os.environ.get("HGEMM_WATCHDOG_CYCLES", "4000000000")
+    # HGEMM_WATCHDOG_CYCLES > 0 builds a debug library whose pipeline waits trap after that
+    # many cycles (a deadlock becomes a launch error instead of a hung GPU).
+    watchdog = os.environ.get("HGEMM_WATCHDOG_CYCLES", "0")
     cmd = [NVCC, *ARCH, f"-DHGEMM_WATCHDOG_CYCLES={watchdog}ll", "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-shared",
            "-I", os.path.join(ROOT, "include"), "-o", tmp, os.path.join(CSRC, "hgemm_api.cu")]
     cmd[1:1] = [f"-D{d}" for d in defines]

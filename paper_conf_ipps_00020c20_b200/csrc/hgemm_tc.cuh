@@ -130,6 +130,68 @@ struct TcShape {
   static_assert(UMMA_N % EPI_COLS == 0, "epilogue chunking");
 };
 
+// Write one thread's 32-word (128-B) row chunk of D: stage it in this warp's
+// swizzled 32 x 128-B box and TMA-store the box, or, for a chunk crossing an N
+// that is not a multiple of 16 B, store it directly (TMA bounds-checks stores
+// at 16-B granularity along the contiguous dimension).
+template <bool OUT_F32, bool CHECK_TAIL = true>
+__device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensorMap *tmD, uint32_t stg,
+                                               uint32_t &nstore, const uint32_t (&w)[32], int col, int row,
+                                               int row_base, uint32_t lane) {
+  constexpr int VEC = OUT_F32 ? 4 : 8;
+  constexpr int COLS = OUT_F32 ? 32 : 64;
+  if (CHECK_TAIL && (p.N & (VEC - 1)) != 0 && col + COLS > p.N) {
+    if (row < p.M) {
+      if constexpr (OUT_F32) {
+        float *dst = static_cast<float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+#pragma unroll
+        for (int j = 0; j < 32; ++j)
+          if (col + j < p.N) dst[j] = __uint_as_float(w[j]);
+      } else {
+        __half *dst = static_cast<__half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const __half2 hv = *reinterpret_cast<const __half2 *>(&w[j]);
+          if (col + 2 * j < p.N) dst[2 * j] = __low2half(hv);
+          if (col + 2 * j + 1 < p.N) dst[2 * j + 1] = __high2half(hv);
+        }
+      }
+    }
+    return;
+  }
+  // stage the 32 x 128-B box (SWIZZLE_128B: 16-B chunk q of row r at q ^ (r % 8))
+  const uint32_t sbuf = stg + (nstore & 1u) * (32u * 128u);
+  if (nstore >= 2) {
+    if (lane == 0) bulk_wait_group_read<1>();  // the store that used this buffer has read it
+    __syncwarp();
+  }
+  const uint32_t rowaddr = sbuf + lane * 128u;
+#pragma unroll
+  for (int q = 0; q < 8; ++q)
+    st_shared_v4(rowaddr + ((q ^ (lane & 7u)) << 4), w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
+  fence_proxy_async_smem();
+  __syncwarp();
+  if (lane == 0) {
+    tma_store_2d(tmD, sbuf, col, row_base);  // the TMA unit clips rows >= M
+    bulk_commit_group();
+  }
+  ++nstore;
+}
+
+// HGEMM_TRACE (experiments only): CTA 0 records clock64 timestamps of the
+// accumulator hand-off into p.probe[8 + 8*tile + field] for its first 16 tiles.
+#ifdef HGEMM_TRACE
+#define HG_TRACE(it, field)                                                              \
+  do {                                                                                   \
+    if (p.probe != nullptr && blockIdx.x == 0 && (it) < 16)                              \
+      p.probe[8 + 8 * (it) + (field)] = static_cast<unsigned long long>(clock64());      \
+  } while (0)
+#else
+#define HG_TRACE(it, field) \
+  do {                      \
+  } while (0)
+#endif
+
 template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32>
 __global__ void __launch_bounds__(192, 1)
     hgemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
@@ -266,6 +328,7 @@ __global__ void __launch_bounds__(192, 1)
         for (int kb = 0; kb < p.num_k_blocks; ++kb) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
+          if (kb == 0) HG_TRACE(it, 6);
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
           const uint32_t sb = sa + A_BYTES;
 #pragma unroll
@@ -275,6 +338,7 @@ __global__ void __launch_bounds__(192, 1)
               if constexpr (CG == 2) mbar_wait_cluster(&tempty[buf * NH + h], acc_phase ^ 1u);
               else mbar_wait(&tempty[buf * NH + h], acc_phase ^ 1u);
               tc_fence_after();
+              HG_TRACE(it, 4 + h);
             }
 #pragma unroll
             for (int k = 0; k < BK / 16; ++k) {
@@ -289,6 +353,7 @@ __global__ void __launch_bounds__(192, 1)
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
         }
         umma_commit<CG>(&tfull[buf]);      // accumulator ready for the epilogue
+        HG_TRACE(it, 0);
       }
     }
   } else {
@@ -304,11 +369,48 @@ __global__ void __launch_bounds__(192, 1)
       tile_coords(t, p, tm, tn);
       const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
       const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
-      mbar_wait_sleep(&tfull[buf], acc_phase);
+      // One thread polls the accumulator barrier; the other epilogue warps
+      // sleep on a named barrier instead of spinning.
+      if (warp == 2 && lane == 0) {
+        mbar_wait(&tfull[buf], acc_phase);
+        HG_TRACE(it, 1);
+      }
+      named_bar_sync(1, 128);
       tc_fence_after();
       const int row_base = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad) * 32;
       const int row = row_base + static_cast<int>(lane);
       const uint32_t tbase = tmem_base + ((quad * 32u) << 16) + buf * BN;
+      if constexpr (!OUT_F32) {
+        if (beta == 0.0f && (p.N & 7) == 0) {
+          // Fast release (FP16 out, beta == 0): read a whole accumulator half into
+          // packed FP16 registers, hand the half back to the MMA warp, then store.
+#pragma unroll 1
+          for (int h = 0; h < NH; ++h) {
+            uint32_t pk[UMMA_N / 2];
+#pragma unroll
+            for (int b = 0; b < UMMA_N / 32; ++b) {
+              uint32_t v[32];
+              tmem_ld_32x32b_x32(tbase + h * UMMA_N + b * 32, v);
+              tmem_ld_wait();
+#pragma unroll
+              for (int j = 0; j < 16; ++j)
+                pk[b * 16 + j] = pack_half2(alpha * __uint_as_float(v[2 * j]), alpha * __uint_as_float(v[2 * j + 1]));
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) {
+              if constexpr (CG == 2) mbar_arrive_cluster(tempty_addr + (buf * NH + h) * 8);
+              else mbar_arrive(&tempty[buf * NH + h]);
+              if (warp == 2) HG_TRACE(it, 2 + h);
+            }
+#pragma unroll
+            for (int c = 0; c < UMMA_N / 64; ++c)
+              emit_row_chunk<false, false>(p, &tmD, stg, nstore, *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
+                                    tn * BN + h * UMMA_N + c * 64, row, row_base, lane);
+          }
+          continue;
+        }
+      }
 #pragma unroll 1
       for (int h = 0; h < NH; ++h) {
 #pragma unroll 1
@@ -325,8 +427,13 @@ __global__ void __launch_bounds__(192, 1)
             if (lane == 0) {
               if constexpr (CG == 2) mbar_arrive_cluster(tempty_addr + (buf * NH + h) * 8);
               else mbar_arrive(&tempty[buf * NH + h]);
+              if (warp == 2) HG_TRACE(it, 2 + h);
             }
           }
+#ifdef HGEMM_EXP_LDONLY
+          if (v[0] == 0x7fc00001u && v[63] == 0x7fc00001u) asm volatile("trap;");  // keep the loads live
+          continue;
+#endif
           // alpha*acc (+ beta*C) in FP32, packed into 32 words = one 128-B row
           uint32_t w[32];
           const int col = tn * BN + colt;
@@ -382,46 +489,7 @@ __global__ void __launch_bounds__(192, 1)
               }
             }
           }
-          // TMA bounds-checks stores at 16-B granularity along the contiguous
-          // dimension: a chunk that crosses an N that is not a multiple of 16 B
-          // (possible only in the last column tile) is written with plain stores.
-          constexpr int VEC = OUT_F32 ? 4 : 8;
-          if ((p.N & (VEC - 1)) != 0 && col + EPI_COLS > p.N) {
-            if (row < p.M) {
-              if constexpr (OUT_F32) {
-                float *dst = static_cast<float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
-#pragma unroll
-                for (int j = 0; j < 32; ++j)
-                  if (col + j < p.N) dst[j] = __uint_as_float(w[j]);
-              } else {
-                __half *dst = static_cast<__half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
-#pragma unroll
-                for (int j = 0; j < 32; ++j) {
-                  const __half2 hv = *reinterpret_cast<const __half2 *>(&w[j]);
-                  if (col + 2 * j < p.N) dst[2 * j] = __low2half(hv);
-                  if (col + 2 * j + 1 < p.N) dst[2 * j + 1] = __high2half(hv);
-                }
-              }
-            }
-            continue;
-          }
-          // stage the 32 x 128-B box (SWIZZLE_128B: 16-B chunk q of row r at q ^ (r % 8))
-          const uint32_t sbuf = stg + (nstore & 1u) * (32u * 128u);
-          if (nstore >= 2) {
-            if (lane == 0) bulk_wait_group_read<1>();  // the store that used this buffer has read it
-            __syncwarp();
-          }
-          const uint32_t rowaddr = sbuf + lane * 128u;
-#pragma unroll
-          for (int q = 0; q < 8; ++q)
-            st_shared_v4(rowaddr + ((q ^ (lane & 7u)) << 4), w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
-          fence_proxy_async_smem();
-          __syncwarp();
-          if (lane == 0) {
-            tma_store_2d(&tmD, sbuf, col, row_base);  // the TMA unit clips rows >= M
-            bulk_commit_group();
-          }
-          ++nstore;
+          emit_row_chunk<OUT_F32>(p, &tmD, stg, nstore, w, col, row, row_base, lane);
         }
       }
     }
