@@ -126,38 +126,68 @@ def max_over_ranks(x, world):
 
 
 # ------------------------------------------------------------------ reference arm (oracle)
+def _oracle_block(workload, ms, ns):
+    """Seeded ms x k op(A) and k x ns op(B) of the workload's shape family, stored with its flags."""
+    from paper_conf_ipps_00020c20_b200 import inputs
+    m, n, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[workload]
+    opA = inputs.uniform_f16(ms, k, 1)
+    opB = inputs.uniform_f16(k, ns, 2)
+    A, lda = inputs.store_op(opA, tA)
+    B, ldb = inputs.store_op(opB, tB)
+    C = inputs.uniform_f16(ms, ns, 3).reshape(-1, order="F") if beta != 0 else None
+    if C is not None and out == "f32":
+        C = C.astype("float32")
+    return (ms, ns, k, alpha, A, lda, B, ldb, beta, C, ms, tA, tB, out)
+
+
+def _time_oracle(workload, ms, ns, threads):
+    import oracle
+    args = _oracle_block(workload, ms, ns)
+    t0 = time.perf_counter()
+    oracle.hgemm_ref(*args, nthreads=threads, want_r=False)
+    return time.perf_counter() - t0
+
+
+def _oracle_sample_size(workload, threads, budget_s):
+    """Grow an ms x ns block (full k) until one oracle call takes about budget_s."""
+    from paper_conf_ipps_00020c20_b200 import inputs
+    m, n, k = inputs.WORKLOADS[workload][:3]
+    ms, ns = min(m, 64), min(n, 64)
+    _time_oracle(workload, ms, ns, threads)                  # warm the threads / page in
+    for _ in range(4):
+        dt = _time_oracle(workload, ms, ns, threads)
+        if dt >= 0.5 * budget_s or (ms == m and ns == n):
+            break
+        f = min(8.0, (budget_s / max(dt, 1e-3)) ** 0.5)
+        ms, ns = max(1, min(m, int(ms * f))), max(1, min(n, int(ns * f)))
+    return ms, ns
+
+
 def run_reference(args, world, rank):
+    """The oracle (the only runnable reference here) on the host cores, on a bounded
+    block of the workload per step; rank 0 only."""
     if rank != 0:
         return 0
-    import numpy as np
     import oracle
     from paper_conf_ipps_00020c20_b200 import inputs
     oracle.build()
     m, n, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[args.workload]
-    sa = inputs.stored_shape(m, k, tA)
-    sb = inputs.stored_shape(k, n, tB)
-    A = inputs.uniform_f16(sa[0], sa[1], 1).reshape(-1, order="F")
-    B = inputs.uniform_f16(sb[0], sb[1], 2).reshape(-1, order="F")
-    C = (inputs.uniform_f16(m, n, 3).reshape(-1, order="F") if beta != 0 else None)
     threads = oracle.max_threads()
-    cols = max(1, min(n, args.ref_cols))
-    # sample: `cols` full columns of C (all m rows), each entry a k-long FP64 dot product
-    ii = np.tile(np.arange(m, dtype=np.int64), cols)
-    jj = np.repeat(np.arange(cols, dtype=np.int64), m)
+    per_step = max(1.0, args.ref_budget / max(1, args.warmup + args.steps))
+    ms, ns = _oracle_sample_size(args.workload, threads, per_step)
     times = []
     for s in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
-        oracle.hgemm_ref_entries(m, n, k, alpha, A, sa[0], B, sb[0], beta, C, m, tA, tB, out, ii, jj,
-                                 nthreads=threads)
-        dt = time.perf_counter() - t0
+        dt = _time_oracle(args.workload, ms, ns, threads)
         if s >= args.warmup:
             times.append(dt)
-    flops = 2.0 * m * cols * k
-    ms = 1e3 * statistics.mean(times)
-    val = flops / (ms * 1e-3) / 1e12
-    sample = f"{cols} full column(s) of C ({m} x {cols} entries, k={k}) of the {m}x{n}x{k} workload per step"
+    flops = 2.0 * ms * ns * k
+    ms_step = 1e3 * statistics.mean(times)
+    val = flops / (ms_step * 1e-3) / 1e12
+    sample = (f"{ms} x {ns} block of C (full k = {k}, layout {tA}{tB}, FP64 oracle) of the {m}x{n}x{k} "
+              f"workload per step")
     line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "strong" if args.workload in inputs.STRONG_SCALING else "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
             "config": {"workload": args.workload, "m": m, "n": n, "k": k, "layout": tA + tB, "out": out},
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
@@ -167,89 +197,78 @@ def run_reference(args, world, rank):
 
 
 def cpu_baseline(workload, budget_s=12.0):
-    """The oracle, as it stands, on the host cores over a bounded sample of the workload."""
-    import numpy as np
+    """The oracle, as it stands, on the host cores over a bounded block of the workload."""
     import oracle
     from paper_conf_ipps_00020c20_b200 import inputs
     oracle.build()
-    m, n, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[workload]
-    sa = inputs.stored_shape(m, k, tA)
-    sb = inputs.stored_shape(k, n, tB)
-    A = inputs.uniform_f16(sa[0], sa[1], 1).reshape(-1, order="F")
-    B = inputs.uniform_f16(sb[0], sb[1], 2).reshape(-1, order="F")
-    C = inputs.uniform_f16(m, n, 3).reshape(-1, order="F") if beta != 0 else None
+    k = inputs.WORKLOADS[workload][2]
     threads = oracle.max_threads()
-    # calibrate on a small sample, then size the timed sample to ~budget_s
-    cnt = 4096
-    g = np.random.Generator(np.random.PCG64(0))
-    ii = g.integers(0, m, cnt)
-    jj = g.integers(0, n, cnt)
-    t0 = time.perf_counter()
-    oracle.hgemm_ref_entries(m, n, k, alpha, A, sa[0], B, sb[0], beta, C, m, tA, tB, out, ii, jj, nthreads=threads)
-    dt = max(time.perf_counter() - t0, 1e-4)
-    cnt = int(min(m * n, max(cnt, cnt * budget_s / dt)))
-    ii = g.integers(0, m, cnt)
-    jj = g.integers(0, n, cnt)
-    t0 = time.perf_counter()
-    oracle.hgemm_ref_entries(m, n, k, alpha, A, sa[0], B, sb[0], beta, C, m, tA, tB, out, ii, jj, nthreads=threads)
-    dt = time.perf_counter() - t0
-    return {"value": 2.0 * cnt * k / dt / 1e12, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": f"{cnt} random entries of C (k={k} FP64 dot products each) of {workload}, {dt:.1f} s"}
+    ms, ns = _oracle_sample_size(workload, threads, budget_s)
+    dt = _time_oracle(workload, ms, ns, threads)
+    return {"value": 2.0 * ms * ns * k / dt / 1e12, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"{ms} x {ns} block of C with the full k = {k} of {workload} ({dt:.1f} s)"}
 
 
 # ------------------------------------------------------------------ our arm
 def run_ours(args, world, rank, local):
     import torch
     from paper_conf_ipps_00020c20_b200 import binding, inputs
-    from paper_conf_ipps_00020c20_b200.sharded import slab_offsets
+    from paper_conf_ipps_00020c20_b200.sharded import broadcast_A, hgemm_sharded, slab_bounds
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=dev)
     lib = binding.load_library()
-    m, n_rank, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[args.workload]
+    m, n_cfg, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[args.workload]
+    strong = args.workload in inputs.STRONG_SCALING
     if args.kernel != "auto":
         binding.set_config(args.kernel, block_n=args.block_n, group_m=args.group_m)
     elif args.group_m:
         binding.set_config("auto", group_m=args.group_m)
-    n_glob = n_rank * world
-    n0 = rank * n_rank
+    # weak scaling: every rank owns an n_cfg-wide slab (global n = n_cfg * world);
+    # strong scaling (config 5): the global n_cfg columns are split over the ranks.
+    n_glob = n_cfg if strong else n_cfg * world
+    n0, n1 = slab_bounds(n_glob, world, rank)
+    n_rank = n1 - n0
     out_t = torch.float32 if out == "f32" else torch.float16
     esz = 4 if out == "f32" else 2
     sa = inputs.stored_shape(m, k, tA)
     sb_rank = inputs.stored_shape(k, n_rank, tB)
-    # device inputs, seeded on the device (bench-only large configs; SURVEY 8(d))
+    # device inputs, seeded on the device (bench-only large configs; SURVEY 8(d)).
+    # Column-major storage: a stored R x C matrix is a (C, R) row-major tensor.
     g = torch.Generator(device=dev).manual_seed(1234)
-    A = (torch.rand(sa[1], sa[0], generator=g, device=dev) * 2 - 1).half()         # column-major storage
+    A = (torch.rand(sa[1], sa[0], generator=g, device=dev) * 2 - 1).half()
     gb = torch.Generator(device=dev).manual_seed(5678 + rank)
-    Bs = (torch.rand(sb_rank[1], sb_rank[0], generator=gb, device=dev) * 2 - 1).half()
-    C = torch.zeros(n_rank, m, dtype=out_t, device=dev)                                # slab, column-major
+    Bs = (torch.rand(sb_rank[1], sb_rank[0], generator=gb, device=dev) * 2 - 1).half()   # this rank's slab
+    C = torch.zeros(n_rank, m, dtype=out_t, device=dev)                                   # this rank's slab
     if beta != 0:
         C.uniform_(-1, 1)
     lda, ldb = sa[0], sb_rank[0]
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
 
-    # collective: replicate A (rank 0's copy) over NCCL, timed separately
+    # the sharded path's one collective: replicate A (rank 0's copy) over NCCL, timed separately
     coll = None
     if world > 1:
         import torch.distributed as dist
         for _ in range(2):
-            dist.broadcast(A, src=0)
+            broadcast_A(A, src=0)
         torch.cuda.synchronize()
         dist.barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        dist.broadcast(A, src=0)
+        broadcast_A(A, src=0)
         e1.record()
         torch.cuda.synchronize()
         bms = max_over_ranks(e0.elapsed_time(e1), world)
-        coll = {"op": "broadcast(A) over NCCL", "bytes": A.numel() * 2, "ms": bms,
-                "GB_s": A.numel() * 2 / (bms * 1e-3) / 1e9}
+        coll = {"op": "broadcast(A) over NCCL (torch.distributed)", "bytes": A.numel() * 2, "ms": bms,
+                "GB_s": A.numel() * 2 / (bms * 1e-3) / 1e9,
+                "note": "reported separately from the GEMM (north_star (3)); not inside value"}
 
     def step():
-        binding.hgemm(m, n_rank, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out, stream.cuda_stream)
+        hgemm_sharded(m, n_glob, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out,
+                      broadcast=False, local_slabs=True, stream=stream.cuda_stream)
 
     for _ in range(args.warmup):
         flush.zero_()
@@ -288,7 +307,8 @@ def run_ours(args, world, rank, local):
     ms_local = statistics.mean(step_ms)
     ms = max_over_ranks(ms_local, world)
     flops_rank = 2.0 * m * n_rank * k
-    value = flops_rank * world / (ms * 1e-3) / 1e12
+    flops_total = 2.0 * m * n_glob * k
+    value = flops_total / (ms * 1e-3) / 1e12
     peaks = load_peaks()
     achieved = flops_rank / (ms_local * 1e-3) / 1e12
     stats = binding.get_stats()
@@ -314,7 +334,7 @@ def run_ours(args, world, rank, local):
         e1.record(stream)
         torch.cuda.synchronize()
         ems = max_over_ranks(e0.elapsed_time(e1) / e2e_steps, world)
-        e2e = {"value": flops_rank * world / (ems * 1e-3) / 1e12, "unit": UNIT,
+        e2e = {"value": flops_total / (ems * 1e-3) / 1e12, "unit": UNIT,
                "h2d_bytes_per_step": (A.numel() + Bs.numel()) * 2 * world,
                "d2h_bytes_per_step": C.numel() * esz * world, "ms_per_step": ems}
 
@@ -365,9 +385,10 @@ def run_ours(args, world, rank, local):
         traffic = load_traffic(args.workload)
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "strong" if strong else "weak",
             "vs_baseline": None, "dtype": "f16xf16->f32 (" + out + " out)", "data": "synthetic",
-            "config": {"workload": args.workload, "m": m, "n": n_glob, "k": k, "n_per_gpu": n_rank,
+            "config": {"workload": args.workload, "m": m, "n": n_glob, "k": k, "n_per_gpu_rank0": n_rank,
                        "layout": tA + tB, "alpha": alpha, "beta": beta, "out": out,
                        "kernel": stats, "l2": "flushed between steps (256 MiB write, outside the events)",
                        "parallelism": f"n-slab x{world}" if world > 1 else "single GPU"},
@@ -402,7 +423,7 @@ def main():
     ap.add_argument("--kernel", default="auto", choices=["auto", "tc1", "tc2", "simt"])
     ap.add_argument("--block-n", type=int, default=0)
     ap.add_argument("--group-m", type=int, default=0)
-    ap.add_argument("--ref-cols", type=int, default=2)
+    ap.add_argument("--ref-budget", type=float, default=60.0, help="seconds of oracle work for --impl reference")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cublas", action="store_true")

@@ -113,7 +113,7 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
     if (CG == 2) {
       cudaLaunchConfig_t qc = {};
       qc.gridDim = dim3(2 * (di.num_sms / 2));
-      qc.blockDim = dim3(192);
+      qc.blockDim = dim3(S::THREADS);
       qc.dynamicSmemBytes = S::SMEM_BYTES;
       cudaLaunchAttribute qa[1];
       qa[0].id = cudaLaunchAttributeClusterDimension;
@@ -136,7 +136,7 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   const int clusters = std::min(tiles, units);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(clusters * CG);
-  cfg.blockDim = dim3(192);
+  cfg.blockDim = dim3(S::THREADS);
   cfg.dynamicSmemBytes = S::SMEM_BYTES;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];

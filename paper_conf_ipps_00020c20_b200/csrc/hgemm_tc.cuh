@@ -24,10 +24,11 @@
 //   SVI-D P:381-397 padded smem layout       -> TMA SWIZZLE_128B + UMMA SW128 descriptors
 //   SIV Eq. 2 P:104 HMMA.1688               -> tcgen05.mma.kind::f16, FP32 accumulation in TMEM
 //
-// Warp roles (192 threads, 1 CTA per SM):
+// Warp roles (320 threads, 1 CTA per SM):
 //   warp 0     : TMA producer (one elected lane)
 //   warp 1     : TMEM allocator; in the leader CTA, the MMA issuer (one lane)
-//   warps 2..5 : epilogue, TMEM lanes 32*(warp%4) .. +31
+//   warps 2..9 : epilogue, TMEM lanes 32*(warp%4) .. +31; warps 2-5 take the first
+//                half of each accumulator half's columns, warps 6-9 the second
 // Pipelines: smem ring full[s]/empty[s]; accumulator hand-off tmem_full[buf] /
 // tmem_empty[buf][half].  BN <= 256 double-buffers the accumulator (epilogue of
 // tile i overlaps the mainloop of tile i+1).  BN = 512 fills TMEM (512 columns)
@@ -47,7 +48,7 @@ struct TcParams {
   int32_t num_m_tiles, num_n_tiles;  // in cluster tiles (128*CG x BN)
   int32_t num_k_blocks;
   int32_t group_m;                   // raster group height, in m-tiles
-  int32_t l2_hint;                   // 0: evict_normal for both; 1: Ak evict_last, Bk evict_first
+  int32_t l2_hint;                   // 0: no hint; 1: Ak evict_last, Bk evict_first; 2: evict_normal
   float alpha, beta;
   void *D;
   int64_t ldd;
@@ -119,22 +120,31 @@ struct TcShape {
   static constexpr int ACC = (2 * BN <= 512) ? 2 : 1;  // accumulator buffers in TMEM
   static constexpr uint32_t TMEM_COLS = (ACC * BN <= 256) ? 256 : 512;
   static constexpr int EPI_COLS = OUT_F32 ? 32 : 64;   // one 128-B staging row per thread
-  static constexpr uint32_t EPI_BYTES = 4 * 2 * 32 * 128;  // 4 warps x 2 buffers x 32 rows x 128 B
+  // 8 epilogue warps: two per TMEM lane quadrant, each owning half of every
+  // accumulator half's columns.  Each warp stages 32 x 128-B boxes in EPI_BUFS
+  // buffers; two buffers when that still leaves >= 4 ring stages.
+  static constexpr int EPI_WARPS = 8;
+  static constexpr int EPI_COLS_W = UMMA_N / 2;        // columns per warp per accumulator half
+  static constexpr int RING_FIT2 =
+      static_cast<int>((227u * 1024u - EPI_WARPS * 2u * 4096u - 2048u) / STAGE_BYTES);
+  static constexpr int EPI_BUFS = RING_FIT2 >= 4 ? 2 : 1;
+  static constexpr uint32_t EPI_BYTES = EPI_WARPS * EPI_BUFS * 32 * 128;
   // As many ring stages as fit in 227 KB next to the staging buffers, barriers and alignment slack.
   static constexpr int STAGES_FIT = static_cast<int>((227u * 1024u - EPI_BYTES - 2048u) / STAGE_BYTES);
   static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
+  static constexpr int THREADS = 64 + 32 * EPI_WARPS;
   static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + EPI_BYTES + 1024 /*barriers*/ + 1024 /*align*/;
   static_assert(BN % 64 == 0 && BN >= 128 && BN <= 512, "BN");
   static_assert(B_ROWS % 64 == 0, "B_ROWS");
   static_assert(STAGES >= 3, "stages");
-  static_assert(UMMA_N % EPI_COLS == 0, "epilogue chunking");
+  static_assert(EPI_COLS_W % EPI_COLS == 0, "epilogue chunking");
 };
 
 // Write one thread's 32-word (128-B) row chunk of D: stage it in this warp's
 // swizzled 32 x 128-B box and TMA-store the box, or, for a chunk crossing an N
 // that is not a multiple of 16 B, store it directly (TMA bounds-checks stores
 // at 16-B granularity along the contiguous dimension).
-template <bool OUT_F32, bool CHECK_TAIL = true>
+template <bool OUT_F32, int EPI_BUFS, bool CHECK_TAIL = true>
 __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensorMap *tmD, uint32_t stg,
                                                uint32_t &nstore, const uint32_t (&w)[32], int col, int row,
                                                int row_base, uint32_t lane) {
@@ -160,9 +170,9 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
     return;
   }
   // stage the 32 x 128-B box (SWIZZLE_128B: 16-B chunk q of row r at q ^ (r % 8))
-  const uint32_t sbuf = stg + (nstore & 1u) * (32u * 128u);
-  if (nstore >= 2) {
-    if (lane == 0) bulk_wait_group_read<1>();  // the store that used this buffer has read it
+  const uint32_t sbuf = stg + (nstore % EPI_BUFS) * (32u * 128u);
+  if (nstore >= EPI_BUFS) {
+    if (lane == 0) bulk_wait_group_read<EPI_BUFS - 1>();  // the store that used this buffer has read it
     __syncwarp();
   }
   const uint32_t rowaddr = sbuf + lane * 128u;
@@ -193,7 +203,7 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
 #endif
 
 template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32>
-__global__ void __launch_bounds__(192, 1)
+__global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     hgemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmD, const TcParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
@@ -206,6 +216,8 @@ __global__ void __launch_bounds__(192, 1)
   constexpr int STAGES = S::STAGES;
   constexpr int ACC = S::ACC;
   constexpr int EPI_COLS = S::EPI_COLS;
+  constexpr int EPI_COLS_W = S::EPI_COLS_W;
+  constexpr int EPI_BUFS = S::EPI_BUFS;
   constexpr uint32_t A_BYTES = S::A_BYTES;
   constexpr uint32_t B_HALF_BYTES = S::B_HALF_BYTES;
   constexpr uint32_t STAGE_BYTES = S::STAGE_BYTES;
@@ -244,7 +256,7 @@ __global__ void __launch_bounds__(192, 1)
       }
       for (int a = 0; a < ACC; ++a) {
         mbar_init(&tfull[a], 1);
-        for (int h = 0; h < NH; ++h) mbar_init(&tempty[a * NH + h], 4 * CG);
+        for (int h = 0; h < NH; ++h) mbar_init(&tempty[a * NH + h], S::EPI_WARPS * CG);
       }
       fence_mbarrier_init();
     }
@@ -266,8 +278,8 @@ __global__ void __launch_bounds__(192, 1)
     if (lane == 0) {
       // Raster groups sweep N with group_m M-tiles held: the Ak panels are
       // re-read by the next waves of the group, the Bk panels only within a wave.
-      const uint64_t pol_a = p.l2_hint == 1 ? l2_policy_evict_last() : l2_policy_evict_normal();
-      const uint64_t pol_b = p.l2_hint == 1 ? l2_policy_evict_first() : l2_policy_evict_normal();
+      const uint64_t pol_a = p.l2_hint == 1 ? l2_policy_evict_last() : p.l2_hint == 2 ? l2_policy_evict_normal() : 0;
+      const uint64_t pol_b = p.l2_hint == 1 ? l2_policy_evict_first() : p.l2_hint == 2 ? l2_policy_evict_normal() : 0;
       uint32_t stage = 0, phase = 0;
       for (int t = cluster_id; t < num_tiles; t += num_clusters) {
         int tm, tn;
@@ -319,37 +331,75 @@ __global__ void __launch_bounds__(192, 1)
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (leader CTA)
     if (rank == 0 && lane == 0) {
+      // For NH == 2 the second accumulator half may still be draining when a
+      // tile starts: half-0 MMAs then run up to MAX_LEAD k-blocks ahead (their
+      // smem stages stay resident) until tempty[half 1] is acquired.
+      constexpr int MAX_LEAD = STAGES - 1;
       uint32_t stage = 0, phase = 0;
       int it = 0;
       for (int t = cluster_id; t < num_tiles; t += num_clusters, ++it) {
         const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
         const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
         const uint32_t d_tmem = tmem_base + buf * BN;
+        bool h1_ready = (NH == 1);
+        int pend_lo = 0;              // first k-block whose half-1 MMAs are not issued yet
+        uint32_t pend_stage = stage;  // its ring stage
         for (int kb = 0; kb < p.num_k_blocks; ++kb) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
-          if (kb == 0) HG_TRACE(it, 6);
-          const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
-          const uint32_t sb = sa + A_BYTES;
-#pragma unroll
-          for (int h = 0; h < NH; ++h) {
-            if (kb == 0) {
-              // this accumulator half must have been drained by the previous tile's epilogue
-              if constexpr (CG == 2) mbar_wait_cluster(&tempty[buf * NH + h], acc_phase ^ 1u);
-              else mbar_wait(&tempty[buf * NH + h], acc_phase ^ 1u);
-              tc_fence_after();
-              HG_TRACE(it, 4 + h);
-            }
-#pragma unroll
-            for (int k = 0; k < BK / 16; ++k) {
-              const uint32_t a_addr = sa + k * A_KSTEP;
-              const uint32_t b_addr = sb + h * B_HALF_BYTES + k * B_KSTEP;
-              const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
-              const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
-              umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
-            }
+          if (kb == 0) {
+            HG_TRACE(it, 6);
+            // accumulator half 0 must have been drained by the previous tile's epilogue
+            if constexpr (CG == 2) mbar_wait_cluster(&tempty[buf * NH], acc_phase ^ 1u);
+            else mbar_wait(&tempty[buf * NH], acc_phase ^ 1u);
+            tc_fence_after();
+            HG_TRACE(it, 4);
           }
-          umma_commit<CG>(&empty[stage]);  // frees the smem stage once these MMAs retire
+          const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            const uint32_t a_addr = sa + k * A_KSTEP;
+            const uint32_t b_addr = sa + A_BYTES + k * B_KSTEP;
+            const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+            const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
+            umma_f16<CG>(d_tmem, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
+          }
+          if constexpr (NH == 2) {
+            if (!h1_ready) {
+              const uint32_t te = smem_u32(&tempty[buf * NH + 1]);
+              if (kb - pend_lo + 1 >= MAX_LEAD || kb == p.num_k_blocks - 1) {
+                if constexpr (CG == 2) mbar_wait_cluster(&tempty[buf * NH + 1], acc_phase ^ 1u);
+                else mbar_wait(&tempty[buf * NH + 1], acc_phase ^ 1u);
+                h1_ready = true;
+              } else {
+                h1_ready = (CG == 2) ? mbar_try_wait_cluster(te, acc_phase ^ 1u) : mbar_try_wait(te, acc_phase ^ 1u);
+              }
+              if (h1_ready) {
+                tc_fence_after();
+                HG_TRACE(it, 5);
+              }
+            }
+            if (h1_ready) {
+              uint32_t s2 = pend_stage;
+              for (int j = pend_lo; j <= kb; ++j) {
+                const uint32_t sa2 = smem_u32(smem + s2 * STAGE_BYTES);
+#pragma unroll
+                for (int k = 0; k < BK / 16; ++k) {
+                  const uint32_t a_addr = sa2 + k * A_KSTEP;
+                  const uint32_t b_addr = sa2 + A_BYTES + B_HALF_BYTES + k * B_KSTEP;
+                  const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+                  const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
+                  umma_f16<CG>(d_tmem + UMMA_N, ad, bd, IDESC, (j | k) != 0 ? 1u : 0u);
+                }
+                umma_commit<CG>(&empty[s2]);  // both halves have consumed this stage
+                if (++s2 == STAGES) s2 = 0;
+              }
+              pend_lo = kb + 1;
+              pend_stage = s2;
+            }
+          } else {
+            umma_commit<CG>(&empty[stage]);  // frees the smem stage once these MMAs retire
+          }
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
         }
         umma_commit<CG>(&tfull[buf]);      // accumulator ready for the epilogue
@@ -358,8 +408,10 @@ __global__ void __launch_bounds__(192, 1)
     }
   } else {
     // ------------------------------------------------------------ epilogue warps
-    const uint32_t quad = warp & 3u;
-    const uint32_t stg = smem_u32(epi_smem) + quad * (2u * 32u * 128u);  // this warp's 2 x 4 KB staging
+    const uint32_t quad = warp & 3u;                 // TMEM lane quadrant this warp may access
+    const uint32_t ew = warp - 2u;                   // epilogue warp index 0..7
+    const int cgrp = static_cast<int>(ew >> 2);      // which half of each accumulator half's columns
+    const uint32_t stg = smem_u32(epi_smem) + ew * (EPI_BUFS * 32u * 128u);
     const uint32_t tempty_addr = (CG == 2) ? mapa_shared(smem_u32(&tempty[0]), 0) : smem_u32(&tempty[0]);
     const float alpha = p.alpha, beta = p.beta;
     uint32_t nstore = 0;
@@ -375,7 +427,7 @@ __global__ void __launch_bounds__(192, 1)
         mbar_wait(&tfull[buf], acc_phase);
         HG_TRACE(it, 1);
       }
-      named_bar_sync(1, 128);
+      named_bar_sync(1, 32 * S::EPI_WARPS);
       tc_fence_after();
       const int row_base = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad) * 32;
       const int row = row_base + static_cast<int>(lane);
@@ -386,11 +438,12 @@ __global__ void __launch_bounds__(192, 1)
           // packed FP16 registers, hand the half back to the MMA warp, then store.
 #pragma unroll 1
           for (int h = 0; h < NH; ++h) {
-            uint32_t pk[UMMA_N / 2];
+            uint32_t pk[EPI_COLS_W / 2];
+            const int c0 = h * UMMA_N + cgrp * EPI_COLS_W;  // first tile column of this warp
 #pragma unroll
-            for (int b = 0; b < UMMA_N / 32; ++b) {
+            for (int b = 0; b < EPI_COLS_W / 32; ++b) {
               uint32_t v[32];
-              tmem_ld_32x32b_x32(tbase + h * UMMA_N + b * 32, v);
+              tmem_ld_32x32b_x32(tbase + c0 + b * 32, v);
               tmem_ld_wait();
 #pragma unroll
               for (int j = 0; j < 16; ++j)
@@ -404,9 +457,10 @@ __global__ void __launch_bounds__(192, 1)
               if (warp == 2) HG_TRACE(it, 2 + h);
             }
 #pragma unroll
-            for (int c = 0; c < UMMA_N / 64; ++c)
-              emit_row_chunk<false, false>(p, &tmD, stg, nstore, *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
-                                    tn * BN + h * UMMA_N + c * 64, row, row_base, lane);
+            for (int c = 0; c < EPI_COLS_W / 64; ++c)
+              emit_row_chunk<false, EPI_BUFS, false>(p, &tmD, stg, nstore,
+                                                     *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
+                                                     tn * BN + c0 + c * 64, row, row_base, lane);
           }
           continue;
         }
@@ -414,13 +468,14 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll 1
       for (int h = 0; h < NH; ++h) {
 #pragma unroll 1
-        for (int c = 0; c < UMMA_N / EPI_COLS; ++c) {
-          const int colt = h * UMMA_N + c * EPI_COLS;  // column within the tile (= TMEM column offset)
+        for (int c = 0; c < EPI_COLS_W / EPI_COLS; ++c) {
+          // column within the tile (= TMEM column offset)
+          const int colt = h * UMMA_N + cgrp * EPI_COLS_W + c * EPI_COLS;
           uint32_t v[64];
           tmem_ld_32x32b_x32(tbase + colt, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
           if constexpr (EPI_COLS == 64) tmem_ld_32x32b_x32(tbase + colt + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
           tmem_ld_wait();
-          if (c == UMMA_N / EPI_COLS - 1) {
+          if (c == EPI_COLS_W / EPI_COLS - 1) {
             // every TMEM read of this half is done: hand it back to the MMA warp
             tc_fence_before();
             __syncwarp();
@@ -489,7 +544,7 @@ __global__ void __launch_bounds__(192, 1)
               }
             }
           }
-          emit_row_chunk<OUT_F32>(p, &tmD, stg, nstore, w, col, row, row_base, lane);
+          emit_row_chunk<OUT_F32, EPI_BUFS>(p, &tmD, stg, nstore, w, col, row, row_base, lane);
         }
       }
     }

@@ -109,7 +109,10 @@ WORKLOADS = {
     "cfg4_skinny_n64": (16384, 64, 4096, "T", "N", 1.0, 0.0, "f16"),
     "cfg4_skinny_n128": (16384, 128, 4096, "T", "N", 1.0, 0.0, "f16"),
     "cfg4_skinny_n256": (16384, 256, 4096, "T", "N", 1.0, 0.0, "f16"),
+    # config 5: the GLOBAL 32768^3 problem, N-slab sharded over the ranks (strong scaling)
+    "cfg5_sharded_32768": (32768, 32768, 32768, "T", "N", 1.0, 0.0, "f16"),
 }
+STRONG_SCALING = {"cfg5_sharded_32768"}
 
 # Square sweep of the paper's evaluation: W = 1024..16384 step 256.
 SQUARE_SWEEP = list(range(1024, 16384 + 1, 256))

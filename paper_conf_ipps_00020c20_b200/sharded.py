@@ -24,6 +24,8 @@ def slab_bounds(n: int, world: int, rank: int, align: int = 8):
     aligned for FP16 when ldc % 8 == 0) except the last one, which is n."""
     if world <= 0 or not (0 <= rank < world):
         raise ValueError("bad world/rank")
+    if n < 0:
+        raise ValueError("n < 0")
     units = (n + align - 1) // align
     base, rem = divmod(units, world)
     u0 = rank * base + min(rank, rem)
@@ -38,27 +40,44 @@ def slab_offsets(n0: int, ldb: int, ldc: int, transB: str, elem_b: int = 2, elem
     return off_b, off_c
 
 
+def _world_rank(group):
+    import torch.distributed as dist
+    if not dist.is_initialized():
+        return 1, 0
+    return dist.get_world_size(group), dist.get_rank(group)
+
+
+def broadcast_A(A, *, group=None, src=0):
+    """Replicate A from rank `src` (the sharded path's one collective)."""
+    import torch.distributed as dist
+    world, _ = _world_rank(group)
+    if world > 1:
+        dist.broadcast(A, src=src, group=group)
+
+
 def hgemm_sharded(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", transB="N",
-                  out_dtype="f16", *, group=None, src=0, broadcast_A=True, gemm=None, stream=None):
+                  out_dtype="f16", *, group=None, src=0, broadcast=True, local_slabs=False,
+                  gemm=None, stream=None):
     """Sharded C = alpha*op(A)*op(B) + beta*C over the ranks of `group`.
 
-    A: the full A tensor on every rank (its contents on rank `src` are
-    broadcast to the others when `broadcast_A`).  B, C: tensors holding the
-    FULL-size column-major storage on this rank (only this rank's slab is
-    read/written), or flat tensors; the slab is addressed by pointer offset.
-    `gemm` defaults to the CUDA hgemm (binding.hgemm); the CPU tests inject
-    another callable with the same signature.  Returns (n0, n1)."""
-    import torch.distributed as dist
-
-    world = dist.get_world_size(group) if dist.is_initialized() else 1
-    rank = dist.get_rank(group) if dist.is_initialized() else 0
-    if broadcast_A and world > 1:
-        dist.broadcast(A, src=src, group=group)
+    n is the GLOBAL number of columns.  A: the full A on every rank (rank
+    `src`'s copy is broadcast first when `broadcast`).  B and C either hold
+    the full-size column-major storage on every rank (local_slabs=False; this
+    rank's slab is addressed by pointer offset) or only this rank's slab
+    (local_slabs=True; the slab starts at the buffer start, same ld).
+    `gemm` defaults to the CUDA hgemm of the C ABI; the CPU tests inject
+    another callable with the same signature.  Returns this rank's (n0, n1)."""
+    world, rank = _world_rank(group)
+    if broadcast:
+        broadcast_A(A, group=group, src=src)
     n0, n1 = slab_bounds(n, world, rank)
     if gemm is None:
         from .binding import hgemm as gemm
     f32 = str(out_dtype) in ("f32", "float32", "torch.float32", "1")
-    off_b, off_c = slab_offsets(n0, ldb, ldc, transB, 2, 4 if f32 else 2)
+    if local_slabs:
+        off_b = off_c = 0
+    else:
+        off_b, off_c = slab_offsets(n0, ldb, ldc, transB, 2, 4 if f32 else 2)
     if n1 > n0:
         gemm(m, n1 - n0, k, alpha, A, lda, _offset(B, off_b), ldb, beta, _offset(C, off_c), ldc,
              transA, transB, out_dtype, stream)
@@ -76,6 +95,8 @@ class _Offset:
 
 
 def _offset(t, off):
+    if off == 0:
+        return t
     if isinstance(t, int):
         return t + off
     return _Offset(t, off)
