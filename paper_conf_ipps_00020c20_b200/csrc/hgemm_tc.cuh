@@ -356,6 +356,26 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
             HG_TRACE(it, 4);
           }
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
+          // Steady state: interleave the halves per K step (consecutive MMAs share
+          // the A descriptor).
+          if (NH == 2 && h1_ready && pend_lo == kb) {
+#pragma unroll
+            for (int k = 0; k < BK / 16; ++k) {
+              const uint32_t a_addr = sa + k * A_KSTEP;
+              const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+#pragma unroll
+              for (int h = 0; h < NH; ++h) {
+                const uint32_t b_addr = sa + A_BYTES + h * B_HALF_BYTES + k * B_KSTEP;
+                const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
+                umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
+              }
+            }
+            umma_commit<CG>(&empty[stage]);
+            pend_lo = kb + 1;
+            if (++pend_stage == STAGES) pend_stage = 0;
+            if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+            continue;
+          }
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
             const uint32_t a_addr = sa + k * A_KSTEP;
