@@ -176,7 +176,7 @@ inline bool is_n(char c) { return c == 'N' || c == 'n'; }
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 // Automatic tile choice: estimated time = waves * per-wave tile cost.
-void choose_tc(int64_t M, int64_t N, int num_sms, int forced_cg, int &cg, int &bn) {
+void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, int forced_cg, int &cg, int &bn) {
   struct Cand { int cg, bn; double eff; };
   // eff: relative per-SM throughput of the tile shape.  Larger tiles move
   // fewer L2->SMEM bytes per FLOP (pair 256x512: 171 FLOP/B, 256x256: 128,
@@ -185,6 +185,11 @@ void choose_tc(int64_t M, int64_t N, int num_sms, int forced_cg, int &cg, int &b
   double best = 1e300;
   for (const Cand &c : cands) {
     if (forced_cg && c.cg != forced_cg) continue;
+    // One 512-column accumulator cannot overlap the epilogue with the next
+    // tile's mainloop; with beta != 0 (C is read in the epilogue) and short K
+    // the exposed epilogue outweighs the bandwidth saving (measured on
+    // BERT-FFN shapes).
+    if (c.bn == 512 && beta_nonzero && K < 4096) continue;
     const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, c.bn);
     const int64_t units = num_sms / c.cg;
     const int64_t waves = cdiv(tiles, units);
@@ -308,7 +313,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   int cg = 2, bn = 512;
   const int forced_cg = cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
   if (forced_cg && cfg.block_n) { cg = forced_cg; bn = cfg.block_n; }
-  else choose_tc(M, N, di.num_sms, forced_cg, cg, bn);
+  else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, cg, bn);
   const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
 
   const bool a_mn = tB;   // Ak = op(B)^T: 'T' -> rows of Ak contiguous along M

@@ -127,7 +127,11 @@ struct TcShape {
   static constexpr int EPI_COLS_W = UMMA_N / 2;        // columns per warp per accumulator half
   static constexpr int RING_FIT2 =
       static_cast<int>((227u * 1024u - EPI_WARPS * 2u * 4096u - 2048u) / STAGE_BYTES);
+#ifdef HGEMM_EPI_BUFS
+  static constexpr int EPI_BUFS = HGEMM_EPI_BUFS;
+#else
   static constexpr int EPI_BUFS = RING_FIT2 >= 4 ? 2 : 1;
+#endif
   static constexpr uint32_t EPI_BYTES = EPI_WARPS * EPI_BUFS * 32 * 128;
   // As many ring stages as fit in 227 KB next to the staging buffers, barriers and alignment slack.
   static constexpr int STAGES_FIT = static_cast<int>((227u * 1024u - EPI_BYTES - 2048u) / STAGE_BYTES);
@@ -182,10 +186,52 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
   fence_proxy_async_smem();
   __syncwarp();
   if (lane == 0) {
+#ifdef HGEMM_C_EVICT_FIRST
+    tma_store_2d_hint(tmD, sbuf, col, row_base, l2_policy_evict_first());
+#else
     tma_store_2d(tmD, sbuf, col, row_base);  // the TMA unit clips rows >= M
+#endif
     bulk_commit_group();
   }
   ++nstore;
+}
+
+// Load COLS FP16 values of C (this thread's row, columns [col, col+COLS)) as
+// COLS/2 packed words; 16-B granules outside [0, N) or rows >= M read as 0.
+// Requires N % 8 == 0 (the fast epilogue path's precondition).
+template <int COLS>
+__device__ __forceinline__ void load_c_words(const TcParams &p, uint32_t (&cw)[COLS / 2], int row, int col) {
+  const __half *src = static_cast<const __half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+#ifdef HGEMM_C_EVICT_FIRST
+  // 32-B loads (N % 8 == 0 and 16-B aligned rows; a 32-B load needs 32-B
+  // alignment, which holds when ldd % 16 == 0 -- otherwise 16-B granules)
+  if ((p.ldd & 15) == 0 && (reinterpret_cast<uintptr_t>(p.D) & 31) == 0) {
+#pragma unroll
+    for (int q = 0; q < COLS / 16; ++q) {
+      uint32_t v[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
+      if (row < p.M && col + 16 * q < p.N) {
+        if (col + 16 * q + 16 <= p.N) {
+          ld_global_v8_evict_first(src + 16 * q, v);
+        } else {
+          const uint4 h = reinterpret_cast<const uint4 *>(src + 16 * q)[0];
+          v[0] = h.x; v[1] = h.y; v[2] = h.z; v[3] = h.w;
+        }
+      }
+#pragma unroll
+      for (int e = 0; e < 8; ++e) cw[8 * q + e] = v[e];
+    }
+    return;
+  }
+#endif
+#pragma unroll
+  for (int q = 0; q < COLS / 8; ++q) {
+    uint4 v = make_uint4(0u, 0u, 0u, 0u);
+    if (row < p.M && col + 8 * q < p.N) v = reinterpret_cast<const uint4 *>(src)[q];
+    cw[4 * q + 0] = v.x;
+    cw[4 * q + 1] = v.y;
+    cw[4 * q + 2] = v.z;
+    cw[4 * q + 3] = v.w;
+  }
 }
 
 // HGEMM_TRACE (experiments only): CTA 0 records clock64 timestamps of the
@@ -344,8 +390,17 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         bool h1_ready = (NH == 1);
         int pend_lo = 0;              // first k-block whose half-1 MMAs are not issued yet
         uint32_t pend_stage = stage;  // its ring stage
+#ifdef HGEMM_TRACE
+        long long full_wait = 0;
+#endif
         for (int kb = 0; kb < p.num_k_blocks; ++kb) {
+#ifdef HGEMM_TRACE
+          const long long tw0 = clock64();
+#endif
           mbar_wait(&full[stage], phase);
+#ifdef HGEMM_TRACE
+          full_wait += clock64() - tw0;
+#endif
           tc_fence_after();
           if (kb == 0) {
             HG_TRACE(it, 6);
@@ -424,6 +479,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         }
         umma_commit<CG>(&tfull[buf]);      // accumulator ready for the epilogue
         HG_TRACE(it, 0);
+#ifdef HGEMM_TRACE
+        if (p.probe != nullptr && blockIdx.x == 0 && it < 16) p.probe[8 + 8 * it + 7] = full_wait;
+#endif
       }
     }
   } else {
@@ -436,11 +494,27 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     const float alpha = p.alpha, beta = p.beta;
     uint32_t nstore = 0;
     int it = 0;
+    // Fast release applies to every case except FP32 output with beta != 0
+    // (whose C half would not fit in registers) and an N that is not a
+    // multiple of 16 B (TMA store granularity).
+    constexpr int VEC = OUT_F32 ? 4 : 8;
+    const bool fast = ((p.N & (VEC - 1)) == 0) && (!OUT_F32 || beta == 0.0f);
+    constexpr int PKW = OUT_F32 ? EPI_COLS_W : EPI_COLS_W / 2;  // packed result words per thread per half
     for (int t = cluster_id; t < num_tiles; t += num_clusters, ++it) {
       int tm, tn;
       tile_coords(t, p, tm, tn);
       const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
       const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
+      const int row_base = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad) * 32;
+      const int row = row_base + static_cast<int>(lane);
+      // FP16 output with beta != 0: this warp's C for accumulator half 0 is
+      // loaded into registers before the accumulator is ready (C does not
+      // depend on it), half 1's while half 0 is being stored.
+      uint32_t cw[OUT_F32 ? 1 : EPI_COLS_W / 2];
+      const bool pre_c = !OUT_F32 && fast && beta != 0.0f;
+      if constexpr (!OUT_F32) {
+        if (pre_c) load_c_words<EPI_COLS_W>(p, cw, row, tn * BN + cgrp * EPI_COLS_W);
+      }
       // One thread polls the accumulator barrier; the other epilogue warps
       // sleep on a named barrier instead of spinning.
       if (warp == 2 && lane == 0) {
@@ -449,41 +523,53 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       }
       named_bar_sync(1, 32 * S::EPI_WARPS);
       tc_fence_after();
-      const int row_base = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad) * 32;
-      const int row = row_base + static_cast<int>(lane);
       const uint32_t tbase = tmem_base + ((quad * 32u) << 16) + buf * BN;
-      if constexpr (!OUT_F32) {
-        if (beta == 0.0f && (p.N & 7) == 0) {
-          // Fast release (FP16 out, beta == 0): read a whole accumulator half into
-          // packed FP16 registers, hand the half back to the MMA warp, then store.
+      if (fast) {
+        // Fast release: read this warp's columns of a whole accumulator half
+        // into registers (alpha, beta*C, FP16 packing applied), hand the half
+        // back to the MMA warp, then store.
 #pragma unroll 1
-          for (int h = 0; h < NH; ++h) {
-            uint32_t pk[EPI_COLS_W / 2];
-            const int c0 = h * UMMA_N + cgrp * EPI_COLS_W;  // first tile column of this warp
+        for (int h = 0; h < NH; ++h) {
+          uint32_t pk[PKW];
+          const int c0 = h * UMMA_N + cgrp * EPI_COLS_W;  // first tile column of this warp
 #pragma unroll
-            for (int b = 0; b < EPI_COLS_W / 32; ++b) {
-              uint32_t v[32];
-              tmem_ld_32x32b_x32(tbase + c0 + b * 32, v);
-              tmem_ld_wait();
+          for (int b = 0; b < EPI_COLS_W / 32; ++b) {
+            uint32_t v[32];
+            tmem_ld_32x32b_x32(tbase + c0 + b * 32, v);
+            tmem_ld_wait();
+            if constexpr (OUT_F32) {
 #pragma unroll
-              for (int j = 0; j < 16; ++j)
-                pk[b * 16 + j] = pack_half2(alpha * __uint_as_float(v[2 * j]), alpha * __uint_as_float(v[2 * j + 1]));
+              for (int j = 0; j < 32; ++j) pk[b * 32 + j] = __float_as_uint(alpha * __uint_as_float(v[j]));
+            } else {
+#pragma unroll
+              for (int j = 0; j < 16; ++j) {
+                float a0 = alpha * __uint_as_float(v[2 * j]), a1 = alpha * __uint_as_float(v[2 * j + 1]);
+                if (pre_c) {
+                  const float2 cf = __half22float2(*reinterpret_cast<const __half2 *>(&cw[b * 16 + j]));
+                  a0 = fmaf(beta, cf.x, a0);
+                  a1 = fmaf(beta, cf.y, a1);
+                }
+                pk[b * 16 + j] = pack_half2(a0, a1);
+              }
             }
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) {
-              if constexpr (CG == 2) mbar_arrive_cluster(tempty_addr + (buf * NH + h) * 8);
-              else mbar_arrive(&tempty[buf * NH + h]);
-              if (warp == 2) HG_TRACE(it, 2 + h);
-            }
-#pragma unroll
-            for (int c = 0; c < EPI_COLS_W / 64; ++c)
-              emit_row_chunk<false, EPI_BUFS, false>(p, &tmD, stg, nstore,
-                                                     *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
-                                                     tn * BN + c0 + c * 64, row, row_base, lane);
           }
-          continue;
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) {
+            if constexpr (CG == 2) mbar_arrive_cluster(tempty_addr + (buf * NH + h) * 8);
+            else mbar_arrive(&tempty[buf * NH + h]);
+            if (warp == 2) HG_TRACE(it, 2 + h);
+          }
+          if constexpr (!OUT_F32) {
+            if (pre_c && h + 1 < NH) load_c_words<EPI_COLS_W>(p, cw, row, tn * BN + (h + 1) * UMMA_N + cgrp * EPI_COLS_W);
+          }
+#pragma unroll
+          for (int c = 0; c < EPI_COLS_W / EPI_COLS; ++c)
+            emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, stg, nstore,
+                                                     *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
+                                                     tn * BN + c0 + c * EPI_COLS, row, row_base, lane);
         }
+        continue;
       }
 #pragma unroll 1
       for (int h = 0; h < NH; ++h) {

@@ -14,28 +14,38 @@ import torch
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_00020c20_b200 import binding  # noqa: E402
 
-m = n = k = int(sys.argv[1]) if len(sys.argv) > 1 else 8192
-bn = int(sys.argv[2]) if len(sys.argv) > 2 else 0
-if bn:
-    binding.set_config("tc2", block_n=bn)
+import argparse  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("m", type=int, nargs="?", default=8192)
+ap.add_argument("--n", type=int, default=0)
+ap.add_argument("--k", type=int, default=0)
+ap.add_argument("--bn", type=int, default=0)
+ap.add_argument("--beta", type=float, default=0.0)
+a = ap.parse_args()
+m = a.m
+n = a.n or m
+k = a.k or m
+if a.bn:
+    binding.set_config("tc2", block_n=a.bn)
 A = (torch.rand(m, k, device="cuda") * 2 - 1).half()
 B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
-C = torch.empty(n, m, dtype=torch.half, device="cuda")
+C = (torch.rand(n, m, device="cuda") * 2 - 1).half()
 probe = torch.zeros(8 + 16 * 8, dtype=torch.int64, device="cuda")
 for i in range(6):
     binding.set_probe(probe if i == 5 else None)
-    binding.hgemm(m, n, k, 1.0, A, k, B, k, 0.0, C, m, "T", "N", "f16")
+    binding.hgemm(m, n, k, 1.0, A, k, B, k, a.beta, C, m, "T", "N", "f16")
 torch.cuda.synchronize()
 v = probe.cpu().tolist()
 t0 = v[0]
 print(f"kernel: {v[2]-v[0]} cycles, {v[3]-v[1]} ns, {(v[2]-v[0])/(v[3]-v[1]):.3f} GHz")
-names = ["mma_done", "epi_wake", "drain0", "drain1", "tempty0", "tempty1", "full0"]
+names = ["mma_done", "epi_wake", "drain0", "drain1", "tempty0", "tempty1", "full0", "fullwait"]
 print("tile " + " ".join(f"{x:>10s}" for x in names))
 for it in range(16):
-    row = v[8 + 8 * it: 8 + 8 * it + 7]
+    row = v[8 + 8 * it: 8 + 8 * it + 8]
     if not any(row):
         break
-    print(f"{it:4d} " + " ".join(f"{(x - t0 if x else 0):10d}" for x in row))
+    print(f"{it:4d} " + " ".join(f"{(x - t0 if x else 0):10d}" for x in row[:7]) + f" {row[7]:10d}")
 for it in range(15):
     a = v[8 + 8 * it: 8 + 8 * it + 7]
     b = v[8 + 8 * (it + 1): 8 + 8 * (it + 1) + 7]
