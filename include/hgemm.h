@@ -80,7 +80,9 @@ typedef enum {
     HGEMM_KERNEL_AUTO = 0,
     HGEMM_KERNEL_SIMT = 1,       /* CUDA-core fallback (always available) */
     HGEMM_KERNEL_TC_1SM = 2,     /* tcgen05 cta_group::1, tile 128 x block_n */
-    HGEMM_KERNEL_TC_2SM = 3      /* tcgen05 cta_group::2 (CTA pair), tile 256 x block_n (256 or 512) */
+    HGEMM_KERNEL_TC_2SM = 3,     /* tcgen05 cta_group::2 (CTA pair), tile 256 x block_n (256 or 512) */
+    HGEMM_KERNEL_SPLITK = 4      /* tcgen05 cta_group::1, tile 128 x block_n (64 or 128), K split over a
+                                    cluster of `splits` CTAs, reduced through distributed shared memory */
 } hgemm_kernel_t;
 
 typedef struct {
@@ -89,6 +91,7 @@ typedef struct {
                           512 (2-SM only); 0 = auto */
     int32_t group_m;   /* L2 raster group height in tiles (0 = auto) */
     int32_t max_ctas;  /* cap on persistent CTAs (0 = all SMs) */
+    int32_t splits;    /* HGEMM_KERNEL_SPLITK: K splits per tile, 2, 4 or 8 (0 = auto) */
 } hgemm_config_t;
 
 /* Set (cfg != NULL) or reset to automatic (cfg == NULL) the process-global

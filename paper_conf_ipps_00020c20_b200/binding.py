@@ -17,7 +17,7 @@ HEADER = os.path.join(_ROOT, "include", "hgemm.h")
 
 HGEMM_OUT_F16 = 0
 HGEMM_OUT_F32 = 1
-HGEMM_KERNEL = {"auto": 0, "simt": 1, "tc1": 2, "tc2": 3}
+HGEMM_KERNEL = {"auto": 0, "simt": 1, "tc1": 2, "tc2": 3, "splitk": 4}
 
 _lib = None
 
@@ -28,7 +28,7 @@ class HgemmError(RuntimeError):
 
 class _Config(ctypes.Structure):
     _fields_ = [("kernel", ctypes.c_int32), ("block_n", ctypes.c_int32),
-                ("group_m", ctypes.c_int32), ("max_ctas", ctypes.c_int32)]
+                ("group_m", ctypes.c_int32), ("max_ctas", ctypes.c_int32), ("splits", ctypes.c_int32)]
 
 
 def lib_path() -> str:
@@ -80,14 +80,15 @@ def _check(code: int):
         raise HgemmError(status_string(code))
 
 
-def set_config(kernel: str | int = "auto", block_n: int = 0, group_m: int = 0, max_ctas: int = 0):
+def set_config(kernel: str | int = "auto", block_n: int = 0, group_m: int = 0, max_ctas: int = 0,
+               splits: int = 0):
     """Force a kernel choice (tests / bench).  ``set_config()`` restores automatic selection."""
     lib = load_library()
     kern = HGEMM_KERNEL[kernel] if isinstance(kernel, str) else int(kernel)
-    if kern == 0 and not block_n and not group_m and not max_ctas:
+    if kern == 0 and not block_n and not group_m and not max_ctas and not splits:
         _check(lib.hgemm_set_config(None))
     else:
-        _check(lib.hgemm_set_config(ctypes.byref(_Config(kern, block_n, group_m, max_ctas))))
+        _check(lib.hgemm_set_config(ctypes.byref(_Config(kern, block_n, group_m, max_ctas, splits))))
 
 
 def set_probe(buf=None):
@@ -107,7 +108,7 @@ def get_stats() -> dict:
     _check(lib.hgemm_get_last_config(ctypes.byref(c)))
     inv = {v: k for k, v in HGEMM_KERNEL.items()}
     return {"last_kernel": inv.get(c.kernel, c.kernel), "block_n": c.block_n, "group_m": c.group_m,
-            "max_ctas": c.max_ctas, "launches": int(lib.hgemm_launch_count())}
+            "max_ctas": c.max_ctas, "splits": c.splits, "launches": int(lib.hgemm_launch_count())}
 
 
 def _ptr(x) -> int:

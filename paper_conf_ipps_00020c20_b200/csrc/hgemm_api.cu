@@ -19,6 +19,7 @@
 
 #include "../../include/hgemm.h"
 #include "hgemm_simt.cuh"
+#include "hgemm_splitk.cuh"
 #include "hgemm_tc.cuh"
 
 namespace {
@@ -37,8 +38,8 @@ constexpr int kMaxDevices = 64;
 DeviceInfo g_dev[kMaxDevices];
 std::mutex g_mu;
 
-hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0};
-hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
+hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
 std::atomic<int64_t> g_launches{0};
 std::atomic<unsigned long long *> g_probe{nullptr};
 
@@ -170,7 +171,87 @@ hgemm_status_t dispatch_tc_layout(bool a_mn, bool b_mn, bool f32, const CUtensor
   return HGEMM_ERR_INVALID_VALUE;
 }
 
+// ----------------------------------------------------------------- split-K launch
+template <int BN, int SPL, bool A_MN, bool B_MN, bool OUT_F32>
+hgemm_status_t launch_splitk(const CUtensorMap &ta, const CUtensorMap &tb, const TcParams &p, int dev,
+                             cudaStream_t stream) {
+  using SH = hg::SkShape<BN, SPL>;
+  auto kern = hg::hgemm_splitk_kernel<BN, SPL, A_MN, B_MN, OUT_F32>;
+  static int attr_done[kMaxDevices] = {};
+  if (!attr_done[dev]) {
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SH::SMEM_BYTES) != cudaSuccess)
+      return HGEMM_ERR_CUDA;
+    if (SPL > 8 && cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess)
+      return HGEMM_ERR_CUDA;
+    attr_done[dev] = 1;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(static_cast<unsigned>(p.num_m_tiles * p.num_n_tiles * SPL));
+  cfg.blockDim = dim3(192);
+  cfg.dynamicSmemBytes = SH::SMEM_BYTES;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = SPL;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (cudaLaunchKernelEx(&cfg, kern, ta, tb, p) != cudaSuccess) return HGEMM_ERR_CUDA;
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+  return HGEMM_SUCCESS;
+}
+
+template <int BN, int SPL>
+hgemm_status_t dispatch_splitk_layout(bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
+                                      const TcParams &p, int dev, cudaStream_t s) {
+#define HG_SK(AM, BM_, F) \
+  if (a_mn == AM && b_mn == BM_ && f32 == F) return launch_splitk<BN, SPL, AM, BM_, F>(ta, tb, p, dev, s);
+  HG_SK(false, false, false)
+  HG_SK(false, false, true)
+  HG_SK(false, true, false)
+  HG_SK(false, true, true)
+  HG_SK(true, false, false)
+  HG_SK(true, false, true)
+  HG_SK(true, true, false)
+  HG_SK(true, true, true)
+#undef HG_SK
+  return HGEMM_ERR_INVALID_VALUE;
+}
+
+hgemm_status_t dispatch_splitk(int bn, int spl, bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta,
+                               const CUtensorMap &tb, const TcParams &p, int dev, cudaStream_t s) {
+  if (bn == 64) {
+    if (spl == 2) return dispatch_splitk_layout<64, 2>(a_mn, b_mn, f32, ta, tb, p, dev, s);
+    if (spl == 4) return dispatch_splitk_layout<64, 4>(a_mn, b_mn, f32, ta, tb, p, dev, s);
+    if (spl == 8) return dispatch_splitk_layout<64, 8>(a_mn, b_mn, f32, ta, tb, p, dev, s);
+  } else {
+    if (spl == 2) return dispatch_splitk_layout<128, 2>(a_mn, b_mn, f32, ta, tb, p, dev, s);
+    if (spl == 4) return dispatch_splitk_layout<128, 4>(a_mn, b_mn, f32, ta, tb, p, dev, s);
+    if (spl == 8) return dispatch_splitk_layout<128, 8>(a_mn, b_mn, f32, ta, tb, p, dev, s);
+  }
+  return HGEMM_ERR_INVALID_VALUE;
+}
+
 inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Split-K choice for under-filled shapes: returns false if the tile grid
+// already fills the GPU.  Cluster sizes of 4 and 8 leave some SMs of a GPC
+// unused (148 SMs do not split into 4-CTA clusters evenly), so the
+// capacity per split count is taken conservatively.
+bool choose_splitk(int64_t M, int64_t N, int64_t K, int num_sms, int &bn, int &spl) {
+  const int64_t nkb = cdiv(K, 64);
+  bn = N <= 64 ? 64 : 128;
+  const int64_t tiles = cdiv(M, 128) * cdiv(N, bn);
+  if (tiles * 2 > num_sms) return false;  // at least half the SMs already busy without splitting
+  spl = 0;
+  const int cands[3] = {8, 4, 2};
+  for (int s : cands) {
+    const int64_t cap = s == 2 ? num_sms : (num_sms * 7) / 8;
+    if (tiles * s <= cap && nkb >= 4 * s) { spl = s; break; }
+  }
+  return spl != 0;
+}
 inline bool is_t(char c) { return c == 'T' || c == 't'; }
 inline bool is_n(char c) { return c == 'N' || c == 'n'; }
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
@@ -215,10 +296,18 @@ const char *hgemm_status_string(hgemm_status_t s) {
 hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!cfg) {
-    g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+    g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
     return HGEMM_SUCCESS;
   }
-  if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_TC_2SM) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_SPLITK) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->kernel == HGEMM_KERNEL_SPLITK) {
+    if (cfg->block_n != 0 && cfg->block_n != 64 && cfg->block_n != 128) return HGEMM_ERR_INVALID_VALUE;
+    if (cfg->splits != 0 && cfg->splits != 2 && cfg->splits != 4 && cfg->splits != 8) return HGEMM_ERR_INVALID_VALUE;
+    if (cfg->group_m < 0 || cfg->max_ctas < 0) return HGEMM_ERR_INVALID_VALUE;
+    g_cfg = *cfg;
+    return HGEMM_SUCCESS;
+  }
+  if (cfg->splits != 0) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->block_n != 0 && cfg->block_n != 128 && cfg->block_n != 256 && cfg->block_n != 512)
     return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_TC_2SM && cfg->block_n == 128) return HGEMM_ERR_INVALID_VALUE;
@@ -255,7 +344,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   if (ldc < std::max<int64_t>(1, m)) return HGEMM_ERR_INVALID_VALUE;
   if (m == 0 || n == 0) {
     std::lock_guard<std::mutex> lk(g_mu);
-    g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+    g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
     return HGEMM_SUCCESS;
   }
   if (!C) return HGEMM_ERR_INVALID_VALUE;
@@ -284,7 +373,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     if (cudaPeekAtLastError() != cudaSuccess) return HGEMM_ERR_CUDA;
     g_launches.fetch_add(1, std::memory_order_relaxed);
     std::lock_guard<std::mutex> lk(g_mu);
-    g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0};
+    g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
     return HGEMM_SUCCESS;
   }
 
@@ -304,20 +393,64 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     if (cudaPeekAtLastError() != cudaSuccess) return HGEMM_ERR_CUDA;
     g_launches.fetch_add(1, std::memory_order_relaxed);
     std::lock_guard<std::mutex> lk(g_mu);
-    g_last = {HGEMM_KERNEL_SIMT, 0, 0, 0};
+    g_last = {HGEMM_KERNEL_SIMT, 0, 0, 0, 0};
     return HGEMM_SUCCESS;
   }
 
   // ---------------------------------------------------------- tcgen05 path
   const int64_t M = n, N = m;  // kernel coordinates (D = C^T)
+  const bool a_mn = tB;   // Ak = op(B)^T: 'T' -> rows of Ak contiguous along M
+  const bool b_mn = !tA;  // Bk = op(A):   'N' -> rows of Bk contiguous along N
+
+  // ---------------------------------------------------------- split-K (under-filled shapes)
+  {
+    int sk_bn = 0, sk_spl = 0;
+    bool use_sk = false;
+    if (cfg.kernel == HGEMM_KERNEL_SPLITK) {
+      use_sk = true;
+      sk_bn = cfg.block_n ? cfg.block_n : (N <= 64 ? 64 : 128);
+      sk_spl = cfg.splits ? cfg.splits : 4;
+    } else if (cfg.kernel == HGEMM_KERNEL_AUTO) {
+      use_sk = choose_splitk(M, N, k, di.num_sms, sk_bn, sk_spl);
+    }
+    if (use_sk) {
+      CUtensorMap ta, tb;
+      bool ok;
+      if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
+      else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
+      if (ok) {
+        if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, sk_bn);
+        else ok = make_map(&tb, A, static_cast<uint64_t>(m), static_cast<uint64_t>(k), lda, 64, 64);
+      }
+      if (!ok) return HGEMM_ERR_CUDA;
+      TcParams p = {};
+      p.M = static_cast<int32_t>(M);
+      p.N = static_cast<int32_t>(N);
+      p.K = static_cast<int32_t>(k);
+      p.num_m_tiles = static_cast<int32_t>(cdiv(M, 128));
+      p.num_n_tiles = static_cast<int32_t>(cdiv(N, sk_bn));
+      p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
+      p.group_m = p.num_m_tiles;  // tiles in m-fastest order
+      p.alpha = alpha;
+      p.beta = beta;
+      p.D = C;
+      p.ldd = ldc;
+      p.probe = nullptr;
+      const hgemm_status_t st = dispatch_splitk(sk_bn, sk_spl, a_mn, b_mn, f32, ta, tb, p, dev, stream);
+      if (st == HGEMM_SUCCESS) {
+        std::lock_guard<std::mutex> lk(g_mu);
+        g_last = {HGEMM_KERNEL_SPLITK, sk_bn, p.group_m, 0, sk_spl};
+      }
+      return st;
+    }
+  }
+
   int cg = 2, bn = 512;
   const int forced_cg = cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
   if (forced_cg && cfg.block_n) { cg = forced_cg; bn = cfg.block_n; }
   else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, cg, bn);
   const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
 
-  const bool a_mn = tB;   // Ak = op(B)^T: 'T' -> rows of Ak contiguous along M
-  const bool b_mn = !tA;  // Bk = op(A):   'N' -> rows of Bk contiguous along N
   CUtensorMap ta, tb;
   bool ok;
   if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
@@ -361,7 +494,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     st = dispatch_tc_layout<128, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);
-    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas};
+    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0};
   }
   return st;
 }

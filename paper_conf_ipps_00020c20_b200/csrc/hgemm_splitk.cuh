@@ -1,0 +1,280 @@
+// Split-K tcgen05 HGEMM for under-filled shapes.
+//
+// Same kernel coordinates as hgemm_tc.cuh (D = C^T row-major, Ak = op(B)^T,
+// Bk = op(A)).  A cluster of S CTAs computes ONE 128 x BN output tile; CTA r
+// of the cluster accumulates k-blocks [r*nkb/S, (r+1)*nkb/S) with
+// tcgen05.mma (cta_group::1) into its own TMEM.  The S partial accumulators
+// are then reduced through distributed shared memory, deterministically:
+// every CTA writes its FP32 partial into its own shared memory, the cluster
+// synchronises, and CTA r sums the column slice [r*BN/S, (r+1)*BN/S) of all
+// S partials in split order 0..S-1 (fixed order => run-to-run bitwise
+// reproducible), applies alpha/beta and stores its slice of D.  No global
+// workspace, no atomics.
+//
+// Paper mapping: the blocked algorithm of Alg. 1 with the K loop
+// (line 6) divided among S thread blocks; the grid of SVI-A.2 is
+// multiplied by S so that shapes with few output tiles (small-batch LSTM
+// gates) still occupy the 148 SMs.
+#pragma once
+#include <cuda_fp16.h>
+
+#include "hgemm_tc.cuh"
+#include "ptx.cuh"
+
+namespace hg {
+
+template <int BN, int S>
+struct SkShape {
+  static constexpr int BM = 128;
+  static constexpr int BK = 64;
+  static constexpr uint32_t A_BYTES = BM * BK * 2;
+  static constexpr uint32_t B_BYTES = BN * BK * 2;
+  static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr uint32_t PART_BYTES = BM * BN * 4;     // FP32 partial accumulator
+  static constexpr int STAGES_FIT = static_cast<int>((227u * 1024u - PART_BYTES - 2048u) / STAGE_BYTES);
+  static constexpr int STAGES = STAGES_FIT > 6 ? 6 : STAGES_FIT;
+  static constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
+  static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + PART_BYTES + 1024 + 1024;
+  static constexpr int SLICE = BN / S;                     // output columns reduced by each CTA
+  static_assert(BN == 64 || BN == 128, "BN");
+  static_assert(S == 2 || S == 4 || S == 8, "S");
+  static_assert(SLICE % 8 == 0, "slice");
+  static_assert(STAGES >= 2, "stages");
+};
+
+// Partial layout in shared memory: row r (TMEM lane) is BN FP32 values =
+// BN/4 16-byte chunks; chunk q of row r is stored at position q ^ (r % 8)
+// within its group of 8 chunks, so 8 consecutive threads (rows) writing the
+// same chunk index hit 8 different 16-byte bank groups.
+__device__ __forceinline__ uint32_t part_off(uint32_t row, uint32_t chunk, uint32_t bn) {
+  const uint32_t q = (chunk & ~7u) | ((chunk ^ row) & 7u);
+  return row * (bn * 4u) + q * 16u;
+}
+
+__device__ __forceinline__ float4 ld_shared_cluster_v4(uint32_t addr) {
+  float4 v;
+  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(addr)
+               : "memory");
+  return v;
+}
+
+template <int BN, int S, bool A_MN, bool B_MN, bool OUT_F32>
+__global__ void __launch_bounds__(192, 1)
+    hgemm_splitk_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                        const TcParams p) {
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
+  using SH = SkShape<BN, S>;
+  constexpr int BM = SH::BM;
+  constexpr int BK = SH::BK;
+  constexpr int STAGES = SH::STAGES;
+  constexpr uint32_t A_BYTES = SH::A_BYTES;
+  constexpr uint32_t STAGE_BYTES = SH::STAGE_BYTES;
+  constexpr uint32_t IDESC = make_idesc_f16<BM, BN, A_MN, B_MN>();
+  constexpr uint32_t A_KSTEP = A_MN ? 16 * 128 : 32;
+  constexpr uint32_t B_KSTEP = B_MN ? 16 * 128 : 32;
+
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw_u32 = smem_u32(smem_raw);
+  uint8_t *smem = smem_raw + ((1024u - (raw_u32 & 1023u)) & 1023u);
+  uint8_t *part = smem + STAGES * STAGE_BYTES;
+  uint64_t *full = reinterpret_cast<uint64_t *>(part + SH::PART_BYTES);
+  uint64_t *empty = full + STAGES;
+  uint64_t *tfull = empty + STAGES;
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tfull + 1);
+
+  const uint32_t warp = warp_id();
+  const uint32_t lane = lane_id();
+  const uint32_t rank = cluster_ctarank();
+  const int tile = static_cast<int>(blockIdx.x) / S;
+  int tm, tn;
+  tile_coords(tile, p, tm, tn);
+  const int kb0 = static_cast<int>((static_cast<int64_t>(p.num_k_blocks) * rank) / S);
+  const int kb1 = static_cast<int>((static_cast<int64_t>(p.num_k_blocks) * (rank + 1)) / S);
+  const int nkb = kb1 - kb0;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+  }
+  if (warp == 1) {
+    if (lane == 0) {
+      for (int s = 0; s < STAGES; ++s) {
+        mbar_init(&full[s], 1);
+        mbar_init(&empty[s], 1);
+      }
+      mbar_init(tfull, 1);
+      fence_mbarrier_init();
+    }
+    __syncwarp();
+    tmem_alloc<1>(smem_u32(tmem_slot), SH::TMEM_COLS);
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------ TMA producer
+    if (lane == 0) {
+      const int a_row = tm * BM;
+      const int b_row = tn * BN;
+      uint32_t stage = 0, phase = 0;
+      for (int kb = kb0; kb < kb1; ++kb) {
+        mbar_wait(&empty[stage], phase ^ 1u);
+        const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
+        const uint32_t sb = sa + A_BYTES;
+        mbar_arrive_expect_tx(&full[stage], STAGE_BYTES);
+        const uint32_t fb = smem_u32(&full[stage]);
+        const int k0 = kb * BK;
+        if constexpr (!A_MN) {
+          tma_load_2d(&tmA, sa, fb, k0, a_row, 0);
+        } else {
+#pragma unroll
+          for (int q = 0; q < BM / 64; ++q) tma_load_2d(&tmA, sa + q * 8192, fb, a_row + 64 * q, k0, 0);
+        }
+        if constexpr (!B_MN) {
+          tma_load_2d(&tmB, sb, fb, k0, b_row, 0);
+        } else {
+#pragma unroll
+          for (int q = 0; q < BN / 64; ++q) tma_load_2d(&tmB, sb + q * 8192, fb, b_row + 64 * q, k0, 0);
+        }
+        if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------ MMA issuer
+    if (lane == 0) {
+      uint32_t stage = 0, phase = 0;
+      for (int j = 0; j < nkb; ++j) {
+        mbar_wait(&full[stage], phase);
+        tc_fence_after();
+        const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
+        const uint32_t sb = sa + A_BYTES;
+#pragma unroll
+        for (int k = 0; k < BK / 16; ++k) {
+          const uint32_t a_addr = sa + k * A_KSTEP;
+          const uint32_t b_addr = sb + k * B_KSTEP;
+          const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+          const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
+          umma_f16<1>(tmem_base, ad, bd, IDESC, (j | k) != 0 ? 1u : 0u);
+        }
+        umma_commit<1>(&empty[stage]);
+        if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+      }
+      if (nkb > 0) umma_commit<1>(tfull);
+      else mbar_arrive(tfull);  // empty K range: the partial is zero
+    }
+  } else {
+    // ------------------------------------------------------------ epilogue warps: partial -> smem
+    const uint32_t quad = warp & 3u;
+    const uint32_t prow = quad * 32u + lane;  // TMEM lane == tile row
+    mbar_wait(tfull, 0);
+    tc_fence_after();
+    const uint32_t pbase = smem_u32(part);
+#pragma unroll
+    for (int c = 0; c < BN / 32; ++c) {
+      uint32_t v[32];
+      if (nkb > 0) {
+        tmem_ld_32x32b_x32(tmem_base + ((quad * 32u) << 16) + c * 32, v);
+        tmem_ld_wait();
+      } else {
+#pragma unroll
+        for (int j = 0; j < 32; ++j) v[j] = 0u;
+      }
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        st_shared_v4(pbase + part_off(prow, c * 8 + q, BN), v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+    }
+    tc_fence_before();
+  }
+
+  // every partial of the cluster is in shared memory
+  cluster_sync();
+
+  if (warp >= 2) {
+    // ------------------------------------------------------------ reduce + epilogue of this CTA's slice
+    constexpr int SLICE = SH::SLICE;
+    const uint32_t quad = warp & 3u;
+    const uint32_t prow = quad * 32u + lane;
+    const int row = tm * BM + static_cast<int>(prow);
+    const int col0 = tn * BN + static_cast<int>(rank) * SLICE;
+    float acc[SLICE];
+#pragma unroll
+    for (int j = 0; j < SLICE; ++j) acc[j] = 0.0f;
+    const uint32_t pbase = smem_u32(part);
+#pragma unroll 1
+    for (int src = 0; src < S; ++src) {  // fixed summation order: split 0, 1, ..., S-1
+      const uint32_t remote = mapa_shared(pbase, static_cast<uint32_t>(src));
+#pragma unroll
+      for (int q = 0; q < SLICE / 4; ++q) {
+        const float4 v = ld_shared_cluster_v4(remote + part_off(prow, rank * (SLICE / 4) + q, BN));
+        acc[4 * q + 0] += v.x;
+        acc[4 * q + 1] += v.y;
+        acc[4 * q + 2] += v.z;
+        acc[4 * q + 3] += v.w;
+      }
+    }
+    if (row < p.M) {
+      const float alpha = p.alpha, beta = p.beta;
+      if constexpr (OUT_F32) {
+        float *dst = static_cast<float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col0;
+#pragma unroll
+        for (int j = 0; j < SLICE; ++j) {
+          if (col0 + j < p.N) {
+            float o = alpha * acc[j];
+            if (beta != 0.0f) o = fmaf(beta, dst[j], o);
+            dst[j] = o;
+          }
+        }
+      } else {
+        __half *dst = static_cast<__half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col0;
+        const bool vec = (col0 + SLICE <= p.N) && ((p.ldd & 7) == 0);
+        if (vec) {
+#pragma unroll
+          for (int q = 0; q < SLICE / 8; ++q) {
+            float f[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) f[e] = alpha * acc[8 * q + e];
+            if (beta != 0.0f) {
+              const uint4 cv = reinterpret_cast<const uint4 *>(dst)[q];
+              const __half2 *ch = reinterpret_cast<const __half2 *>(&cv);
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const float2 cf = __half22float2(ch[e]);
+                f[2 * e] = fmaf(beta, cf.x, f[2 * e]);
+                f[2 * e + 1] = fmaf(beta, cf.y, f[2 * e + 1]);
+              }
+            }
+            uint4 o;
+            o.x = pack_half2(f[0], f[1]);
+            o.y = pack_half2(f[2], f[3]);
+            o.z = pack_half2(f[4], f[5]);
+            o.w = pack_half2(f[6], f[7]);
+            reinterpret_cast<uint4 *>(dst)[q] = o;
+          }
+        } else {
+#pragma unroll
+          for (int j = 0; j < SLICE; ++j) {
+            if (col0 + j < p.N) {
+              float o = alpha * acc[j];
+              if (beta != 0.0f) o = fmaf(beta, __half2float(dst[j]), o);
+              dst[j] = __float2half_rn(o);
+            }
+          }
+        }
+      }
+    }
+  }
+
+  // peers must not exit while their shared memory is being read
+  cluster_sync();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<1>(tmem_base, SH::TMEM_COLS);
+  }
+#endif
+}
+
+}  // namespace hg

@@ -18,7 +18,8 @@ from .gpu_util import GpuCase, assert_within_tolerance, ulp16
 pytestmark = pytest.mark.gpu
 
 TRANS = [("N", "N"), ("N", "T"), ("T", "N"), ("T", "T")]
-KERNELS = [("tc2", 512), ("tc2", 256), ("tc1", 256), ("tc1", 128), ("simt", 0)]
+KERNELS = [("tc2", 512), ("tc2", 256), ("tc1", 256), ("tc1", 128), ("splitk", 64), ("splitk", 128), ("simt", 0)]
+TC_KERNELS = KERNELS[:4]   # same K order inside the tensor core -> bitwise identical results
 
 
 @pytest.fixture(autouse=True)
@@ -197,7 +198,7 @@ def test_all_kernels_agree_on_random(oracle_mod):
     order inside the tensor core, so tc1/tc2 results are bitwise identical."""
     m, n, k = 700, 900, 640
     base = None
-    for kernel, bn in KERNELS[:4]:
+    for kernel, bn in TC_KERNELS:
         _use(kernel, bn)
         case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", out="f32")
         got = case.run_gpu()
@@ -205,3 +206,38 @@ def test_all_kernels_agree_on_random(oracle_mod):
             base = got
         else:
             assert np.array_equal(got.view(np.uint32), base.view(np.uint32)), kernel
+
+
+@pytest.mark.parametrize("splits", [2, 4, 8])
+@pytest.mark.parametrize("bn", [64, 128])
+@pytest.mark.parametrize("tA,tB", TRANS)
+def test_splitk_splits(oracle_mod, splits, bn, tA, tB):
+    """Split-K over a cluster: every split count, ragged K ranges (some splits empty)."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("splitk", block_n=bn, splits=splits)
+    for (m, n, k) in [(200, 300, 1000), (64, 4096, 448), (130, 257, 100)]:
+        case = GpuCase(inputs.uniform_f16(m, k, 7), inputs.uniform_f16(k, n, 8), tA, tB, 1.0, 0.5,
+                       C=inputs.uniform_f16(m, n, 9), out="f16")
+        got = case.run_gpu()
+        assert case.stats["last_kernel"] == "splitk" and case.stats["splits"] == splits, case.stats
+        _, r, ab = case.oracle(oracle_mod)
+        assert_within_tolerance(case, got, r, ab)
+        a, b = case.run_gpu(repeat=2)
+        assert np.array_equal(a.view(np.uint16), b.view(np.uint16))   # deterministic reduction order
+    opA = inputs.integer_f16(90, 640, 3, -4, 4)
+    opB = inputs.integer_f16(640, 70, 4, -4, 4)
+    case = GpuCase(opA, opB, tA, tB, out="f32")
+    got = case.view(case.run_gpu())
+    _, r, _ = case.oracle(oracle_mod)
+    assert np.array_equal(got.astype(np.float64), r)
+
+
+def test_splitk_auto_for_underfilled(oracle_mod):
+    """LSTM-gate shape (m=64 batch, n=4096, k=2048): automatic selection splits K."""
+    m, n, k = 64, 4096, 2048
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", 1.0, 1.0,
+                   C=inputs.uniform_f16(m, n, 3), out="f16")
+    got = case.run_gpu()
+    assert case.stats["last_kernel"] == "splitk", case.stats
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, got, r, ab)
