@@ -435,7 +435,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
       p.beta = beta;
       p.D = C;
       p.ldd = ldc;
-      p.probe = nullptr;
+      p.probe = g_probe.load(std::memory_order_relaxed);
       const hgemm_status_t st = dispatch_splitk(sk_bn, sk_spl, a_mn, b_mn, f32, ta, tb, p, dev, stream);
       if (st == HGEMM_SUCCESS) {
         std::lock_guard<std::mutex> lk(g_mu);

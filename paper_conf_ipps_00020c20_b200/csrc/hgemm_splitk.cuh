@@ -5,11 +5,12 @@
 // of the cluster accumulates k-blocks [r*nkb/S, (r+1)*nkb/S) with
 // tcgen05.mma (cta_group::1) into its own TMEM.  The S partial accumulators
 // are then reduced through distributed shared memory, deterministically:
-// every CTA writes its FP32 partial into its own shared memory, the cluster
-// synchronises, and CTA r sums the column slice [r*BN/S, (r+1)*BN/S) of all
-// S partials in split order 0..S-1 (fixed order => run-to-run bitwise
-// reproducible), applies alpha/beta and stores its slice of D.  No global
-// workspace, no atomics.
+// CTA r owns the column slice [r*BN/S, (r+1)*BN/S); every CTA pushes each
+// slice of its FP32 partial into the owner's shared memory (remote
+// st.shared::cluster), the cluster synchronises once, and each owner sums
+// its S received slices in split order 0..S-1 (fixed order => run-to-run
+// bitwise reproducible), applies alpha/beta and stores its slice of D.  No
+// global workspace, no atomics.
 //
 // Paper mapping: the blocked algorithm of Alg. 1 with the K loop
 // (line 6) divided among S thread blocks; the grid of SVI-A.2 is
@@ -30,7 +31,7 @@ struct SkShape {
   static constexpr uint32_t A_BYTES = BM * BK * 2;
   static constexpr uint32_t B_BYTES = BN * BK * 2;
   static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr uint32_t PART_BYTES = BM * BN * 4;     // FP32 partial accumulator
+  static constexpr uint32_t PART_BYTES = BM * BN * 4;     // receive buffer: S x 128 rows x BN/S FP32
   static constexpr int STAGES_FIT = static_cast<int>((227u * 1024u - PART_BYTES - 2048u) / STAGE_BYTES);
   static constexpr int STAGES = STAGES_FIT > 6 ? 6 : STAGES_FIT;
   static constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
@@ -42,13 +43,26 @@ struct SkShape {
   static_assert(STAGES >= 2, "stages");
 };
 
-// Partial layout in shared memory: row r (TMEM lane) is BN FP32 values =
-// BN/4 16-byte chunks; chunk q of row r is stored at position q ^ (r % 8)
-// within its group of 8 chunks, so 8 consecutive threads (rows) writing the
-// same chunk index hit 8 different 16-byte bank groups.
-__device__ __forceinline__ uint32_t part_off(uint32_t row, uint32_t chunk, uint32_t bn) {
-  const uint32_t q = (chunk & ~7u) | ((chunk ^ row) & 7u);
-  return row * (bn * 4u) + q * 16u;
+// Receive buffer of the owner CTA: [S sources][128 rows][SLICE FP32], the
+// 16-byte chunk index of a row rotated by the row so that consecutive rows
+// (threads) writing or reading the same chunk use different bank groups.
+template <int SLICE>
+__device__ __forceinline__ uint32_t recv_off_t(uint32_t src, uint32_t row, uint32_t chunk) {
+  constexpr uint32_t CH = SLICE / 4;                      // 16-byte chunks per row
+  const uint32_t q = (chunk + row) % CH;
+  return (src * 128u + row) * (SLICE * 4u) + q * 16u;
+}
+
+__device__ __forceinline__ void st_shared_cluster_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t c,
+                                                     uint32_t d) {
+  asm volatile("st.shared::cluster.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d)
+               : "memory");
+}
+__device__ __forceinline__ float4 ld_shared_f4(uint32_t addr) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(addr)
+               : "memory");
+  return v;
 }
 
 __device__ __forceinline__ float4 ld_shared_cluster_v4(uint32_t addr) {
@@ -93,7 +107,42 @@ __global__ void __launch_bounds__(192, 1)
   const int kb0 = static_cast<int>((static_cast<int64_t>(p.num_k_blocks) * rank) / S);
   const int kb1 = static_cast<int>((static_cast<int64_t>(p.num_k_blocks) * (rank + 1)) / S);
   const int nkb = kb1 - kb0;
+  auto recv_off = [](uint32_t src, uint32_t row, uint32_t chunk) { return recv_off_t<SH::SLICE>(src, row, chunk); };
 
+#ifdef HGEMM_TRACE
+#define SK_TRACE(f)                                                                            \
+  do {                                                                                         \
+    if (p.probe != nullptr && blockIdx.x < 256) p.probe[8 + 8 * blockIdx.x + (f)] = globaltimer_ns(); \
+  } while (0)
+#else
+#define SK_TRACE(f) \
+  do {              \
+  } while (0)
+#endif
+  if (threadIdx.x == 0) SK_TRACE(0);
+  // Epilogue warps prefetch their C slice (FP16 vector path, beta != 0) at
+  // kernel start: C does not depend on the accumulator.
+  uint32_t cpre[SH::SLICE / 2];
+#pragma unroll
+  for (int j = 0; j < SH::SLICE / 2; ++j) cpre[j] = 0u;
+  if constexpr (!OUT_F32) {
+    if (warp >= 2 && p.beta != 0.0f) {
+      const int row = tm * BM + static_cast<int>((warp & 3u) * 32u + lane);
+      const int col0 = tn * BN + static_cast<int>(rank) * SH::SLICE;
+      if (row < p.M && col0 + SH::SLICE <= p.N && (p.ldd & 7) == 0) {
+        const uint4 *src = reinterpret_cast<const uint4 *>(static_cast<const __half *>(p.D) +
+                                                          static_cast<int64_t>(row) * p.ldd + col0);
+#pragma unroll
+        for (int q = 0; q < SH::SLICE / 8; ++q) {
+          const uint4 v = src[q];
+          cpre[4 * q] = v.x;
+          cpre[4 * q + 1] = v.y;
+          cpre[4 * q + 2] = v.z;
+          cpre[4 * q + 3] = v.w;
+        }
+      }
+    }
+  }
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
@@ -114,6 +163,7 @@ __global__ void __launch_bounds__(192, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (threadIdx.x == 0) SK_TRACE(1);
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer
@@ -150,6 +200,7 @@ __global__ void __launch_bounds__(192, 1)
       for (int j = 0; j < nkb; ++j) {
         mbar_wait(&full[stage], phase);
         tc_fence_after();
+        if (j == 0) SK_TRACE(2);
         const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
         const uint32_t sb = sa + A_BYTES;
 #pragma unroll
@@ -163,16 +214,22 @@ __global__ void __launch_bounds__(192, 1)
         umma_commit<1>(&empty[stage]);
         if (++stage == STAGES) { stage = 0; phase ^= 1u; }
       }
+      SK_TRACE(3);
       if (nkb > 0) umma_commit<1>(tfull);
       else mbar_arrive(tfull);  // empty K range: the partial is zero
     }
   } else {
-    // ------------------------------------------------------------ epilogue warps: partial -> smem
+    // ------------------------------------------------------------ epilogue warps: push partial slices
+    // CTA `rank` owns output columns [rank*SLICE, (rank+1)*SLICE) of the tile.
+    // Each CTA pushes the slice owned by CTA o into o's receive buffer at
+    // [rank][row][0..SLICE) (remote shared-memory stores, posted), so after
+    // one cluster barrier every owner reduces from its local shared memory.
     const uint32_t quad = warp & 3u;
     const uint32_t prow = quad * 32u + lane;  // TMEM lane == tile row
     mbar_wait(tfull, 0);
     tc_fence_after();
-    const uint32_t pbase = smem_u32(part);
+    if (warp == 2 && lane == 0) SK_TRACE(4);
+    const uint32_t rbuf = smem_u32(part);
 #pragma unroll
     for (int c = 0; c < BN / 32; ++c) {
       uint32_t v[32];
@@ -184,32 +241,37 @@ __global__ void __launch_bounds__(192, 1)
         for (int j = 0; j < 32; ++j) v[j] = 0u;
       }
 #pragma unroll
-      for (int q = 0; q < 8; ++q)
-        st_shared_v4(pbase + part_off(prow, c * 8 + q, BN), v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+      for (int q = 0; q < 8; ++q) {
+        const int colq = c * 32 + 4 * q;                  // first of these 4 tile columns
+        const uint32_t owner = static_cast<uint32_t>(colq / SH::SLICE);
+        const uint32_t within = static_cast<uint32_t>(colq % SH::SLICE) / 4;  // 16-B chunk in the slice
+        const uint32_t dst = mapa_shared(rbuf + recv_off(rank, prow, within), owner);
+        st_shared_cluster_v4(dst, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+      }
     }
     tc_fence_before();
   }
 
-  // every partial of the cluster is in shared memory
+  // every slice has been pushed to its owner
   cluster_sync();
+  if (threadIdx.x == 0) SK_TRACE(5);
 
   if (warp >= 2) {
-    // ------------------------------------------------------------ reduce + epilogue of this CTA's slice
+    // ------------------------------------------------------------ local reduce + epilogue of this CTA's slice
     constexpr int SLICE = SH::SLICE;
     const uint32_t quad = warp & 3u;
     const uint32_t prow = quad * 32u + lane;
     const int row = tm * BM + static_cast<int>(prow);
     const int col0 = tn * BN + static_cast<int>(rank) * SLICE;
+    const uint32_t rbuf = smem_u32(part);
     float acc[SLICE];
 #pragma unroll
     for (int j = 0; j < SLICE; ++j) acc[j] = 0.0f;
-    const uint32_t pbase = smem_u32(part);
-#pragma unroll 1
+#pragma unroll
     for (int src = 0; src < S; ++src) {  // fixed summation order: split 0, 1, ..., S-1
-      const uint32_t remote = mapa_shared(pbase, static_cast<uint32_t>(src));
 #pragma unroll
       for (int q = 0; q < SLICE / 4; ++q) {
-        const float4 v = ld_shared_cluster_v4(remote + part_off(prow, rank * (SLICE / 4) + q, BN));
+        const float4 v = ld_shared_f4(rbuf + recv_off(static_cast<uint32_t>(src), prow, q));
         acc[4 * q + 0] += v.x;
         acc[4 * q + 1] += v.y;
         acc[4 * q + 2] += v.z;
@@ -238,8 +300,7 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll
             for (int e = 0; e < 8; ++e) f[e] = alpha * acc[8 * q + e];
             if (beta != 0.0f) {
-              const uint4 cv = reinterpret_cast<const uint4 *>(dst)[q];
-              const __half2 *ch = reinterpret_cast<const __half2 *>(&cv);
+              const __half2 *ch = reinterpret_cast<const __half2 *>(&cpre[4 * q]);
 #pragma unroll
               for (int e = 0; e < 4; ++e) {
                 const float2 cf = __half22float2(ch[e]);
@@ -268,8 +329,10 @@ __global__ void __launch_bounds__(192, 1)
     }
   }
 
+  if (threadIdx.x == 64) SK_TRACE(6);
   // peers must not exit while their shared memory is being read
   cluster_sync();
+  if (threadIdx.x == 0) SK_TRACE(7);
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc<1>(tmem_base, SH::TMEM_COLS);
