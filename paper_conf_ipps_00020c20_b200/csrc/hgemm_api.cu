@@ -471,8 +471,12 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   p.num_m_tiles = static_cast<int32_t>(cdiv(M, 128 * cg));
   p.num_n_tiles = static_cast<int32_t>(cdiv(N, bn));
   p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
-  p.group_m = cfg.group_m > 0 ? cfg.group_m : 8;
+  p.group_m = cfg.group_m > 0 ? cfg.group_m : 16;  // measured best with 256x512 pair tiles (profiles/)
   p.group_m = std::max(1, std::min(p.group_m, p.num_m_tiles));
+  if (const char *e = std::getenv("HGEMM_GROUP_N")) {  // experiments: group along N instead
+    const int gn = std::atoi(e);
+    if (gn > 0) p.group_m = -std::max(1, std::min(gn, p.num_n_tiles));
+  }
   {
     const char *e = std::getenv("HGEMM_L2_HINT");
     p.l2_hint = e ? std::atoi(e) : 0;

@@ -47,7 +47,7 @@ struct TcParams {
   int32_t M, N, K;                   // D is M x N, reduction length K
   int32_t num_m_tiles, num_n_tiles;  // in cluster tiles (128*CG x BN)
   int32_t num_k_blocks;
-  int32_t group_m;                   // raster group height, in m-tiles
+  int32_t group_m;                   // raster group height in m-tiles (> 0), or width in n-tiles (< 0)
   int32_t l2_hint;                   // 0: no hint; 1: Ak evict_last, Bk evict_first; 2: evict_normal
   float alpha, beta;
   void *D;
@@ -92,6 +92,18 @@ __host__ __device__ constexpr uint32_t make_idesc_f16() {
 }
 
 __device__ __forceinline__ void tile_coords(int t, const TcParams &p, int &tm, int &tn) {
+  if (p.group_m < 0) {
+    // grouped along N: -group_m n-tiles per group, n fastest
+    const int gn = -p.group_m;
+    const int per_group = gn * p.num_m_tiles;
+    const int g = t / per_group;
+    const int first_n = g * gn;
+    const int gsz = min(p.num_n_tiles - first_n, gn);
+    const int r = t - g * per_group;
+    tn = first_n + r % gsz;
+    tm = r / gsz;
+    return;
+  }
   const int per_group = p.group_m * p.num_n_tiles;
   const int g = t / per_group;
   const int first_m = g * p.group_m;
