@@ -17,6 +17,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libhgemm.so")
+MB_LIB = os.path.join(PKG, "libhgemm_mb.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -53,8 +54,28 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     return target
 
 
+def build_microbench(force: bool = False) -> str:
+    """The B200 micro-benchmark library (csrc/microbench.cu; NEXT-4, not on the GEMM path)."""
+    src = os.path.join(CSRC, "microbench.cu")
+    deps = [src] + glob.glob(os.path.join(CSRC, "*.cuh"))
+    if not force and os.path.exists(MB_LIB) and all(os.path.getmtime(d) <= os.path.getmtime(MB_LIB) for d in deps):
+        return MB_LIB
+    tmp = MB_LIB + f".tmp{os.getpid()}"
+    subprocess.check_call([NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
+                           "-o", tmp, src])
+    os.replace(tmp, MB_LIB)
+    return MB_LIB
+
+
+def build_all(force: bool = False) -> None:
+    build(force=force)
+    build_microbench(force=force)
+
+
 if __name__ == "__main__":
     defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
     outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
     print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv, defines=defs,
                 out=outs[0] if outs else None))
+    if "--microbench" in sys.argv:
+        print(build_microbench(force="--force" in sys.argv))

@@ -252,7 +252,7 @@ __device__ __forceinline__ void load_c_words(const TcParams &p, uint32_t (&cw)[C
 #define HG_TRACE(it, field)                                                              \
   do {                                                                                   \
     if (p.probe != nullptr && blockIdx.x == 0 && (it) < 16)                              \
-      p.probe[8 + 8 * (it) + (field)] = static_cast<unsigned long long>(clock64());      \
+      p.probe[8 + 16 * (it) + (field)] = static_cast<unsigned long long>(clock64());     \
   } while (0)
 #else
 #define HG_TRACE(it, field) \
@@ -492,7 +492,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         umma_commit<CG>(&tfull[buf]);      // accumulator ready for the epilogue
         HG_TRACE(it, 0);
 #ifdef HGEMM_TRACE
-        if (p.probe != nullptr && blockIdx.x == 0 && it < 16) p.probe[8 + 8 * it + 7] = full_wait;
+        if (p.probe != nullptr && blockIdx.x == 0 && it < 16) p.probe[8 + 16 * it + 7] = full_wait;
 #endif
       }
     }
@@ -535,6 +535,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       }
       named_bar_sync(1, 32 * S::EPI_WARPS);
       tc_fence_after();
+      if (warp == 2 && lane == 0) HG_TRACE(it, 8);
       const uint32_t tbase = tmem_base + ((quad * 32u) << 16) + buf * BN;
       if (fast) {
         // Fast release: read this warp's columns of a whole accumulator half
@@ -544,6 +545,25 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         for (int h = 0; h < NH; ++h) {
           uint32_t pk[PKW];
           const int c0 = h * UMMA_N + cgrp * EPI_COLS_W;  // first tile column of this warp
+          if (!pre_c) {
+            // two TMEM loads in flight per wait (no C registers live in this case)
+#pragma unroll
+            for (int b = 0; b < EPI_COLS_W / 64; ++b) {
+              uint32_t v[64];
+              tmem_ld_32x32b_x32(tbase + c0 + b * 64, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+              tmem_ld_32x32b_x32(tbase + c0 + b * 64 + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+              tmem_ld_wait();
+              if (warp == 2 && lane == 0 && h == 0 && b == 0) HG_TRACE(it, 9);
+              if constexpr (OUT_F32) {
+#pragma unroll
+                for (int j = 0; j < 64; ++j) pk[b * 64 + j] = __float_as_uint(alpha * __uint_as_float(v[j]));
+              } else {
+#pragma unroll
+                for (int j = 0; j < 32; ++j)
+                  pk[b * 32 + j] = pack_half2(alpha * __uint_as_float(v[2 * j]), alpha * __uint_as_float(v[2 * j + 1]));
+              }
+            }
+          } else
 #pragma unroll
           for (int b = 0; b < EPI_COLS_W / 32; ++b) {
             uint32_t v[32];
@@ -565,11 +585,13 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
               }
             }
           }
+          if (warp == 2 && lane == 0) HG_TRACE(it, 10 + h);
           tc_fence_before();
           __syncwarp();
           if (lane == 0) {
-            if constexpr (CG == 2) mbar_arrive_cluster(tempty_addr + (buf * NH + h) * 8);
-            else mbar_arrive(&tempty[buf * NH + h]);
+            // TMEM reads are complete (tcgen05.wait::ld): a relaxed arrival suffices
+            if constexpr (CG == 2) mbar_arrive_cluster_relaxed(tempty_addr + (buf * NH + h) * 8);
+            else mbar_arrive_relaxed(&tempty[buf * NH + h]);
             if (warp == 2) HG_TRACE(it, 2 + h);
           }
           if constexpr (!OUT_F32) {
@@ -598,8 +620,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
             tc_fence_before();
             __syncwarp();
             if (lane == 0) {
-              if constexpr (CG == 2) mbar_arrive_cluster(tempty_addr + (buf * NH + h) * 8);
-              else mbar_arrive(&tempty[buf * NH + h]);
+              if constexpr (CG == 2) mbar_arrive_cluster_relaxed(tempty_addr + (buf * NH + h) * 8);
+              else mbar_arrive_relaxed(&tempty[buf * NH + h]);
               if (warp == 2) HG_TRACE(it, 2 + h);
             }
           }

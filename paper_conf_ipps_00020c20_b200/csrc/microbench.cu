@@ -1,0 +1,252 @@
+// B200 (sm_100a) micro-benchmarks: the paper's SIV-SV characterisation
+// ("demystifying" the tensor core and the memory hierarchy, PAPER.md
+// P:156-238, Tables I-V) redone for the units the tcgen05 HGEMM uses
+// (SURVEY 8(f) NEXT-4).  Separate library (libhgemm_mb.so), not on the
+// GEMM path; driven by tools/microbench.py.
+//
+//   mb_mma_rate   : tcgen05.mma kind::f16 issue-to-completion throughput
+//                   (cycles per instruction) for cta_group::1 M=128 and
+//                   cta_group::2 M=256, N in {64,128,256}; the analogue of
+//                   Table I's HMMA.1688 CPI.
+//   mb_mma_latency: one tcgen05.mma + tcgen05.commit -> mbarrier round trip.
+//   mb_tmem_ld    : tcgen05.ld 32x32b.x32 bytes/cycle per SM with 4 or 8 warps.
+//   mb_tma_load   : TMA (cp.async.bulk.tensor) bytes/cycle per SM and chip
+//                   GB/s, from an L2-resident tile and streaming from HBM;
+//                   the analogue of Table II / Table III.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "hgemm_tc.cuh"
+
+namespace mb {
+using namespace hg;
+
+// ------------------------------------------------------------------ MMA throughput / latency
+template <int CG, int N>
+__global__ void __launch_bounds__(128, 1) mma_rate_kernel(int iters, unsigned long long *out, int latency_mode) {
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
+  constexpr int M = 128 * CG;
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  uint8_t *smem = smem_raw + ((1024u - (raw & 1023u)) & 1023u);
+  // operands: A 128 x 64 FP16 (16 KB) and B (N/CG) x 64 FP16, K-major SW128; contents irrelevant
+  uint64_t *bar = reinterpret_cast<uint64_t *>(smem + 16384 + (N / CG) * 128);
+  uint32_t *slot = reinterpret_cast<uint32_t *>(bar + 1);
+  const uint32_t warp = warp_id(), lane = lane_id();
+  const uint32_t rank = CG == 2 ? cluster_ctarank() : 0u;
+  if (warp == 0) {
+    if (lane == 0) {
+      mbar_init(bar, 1);
+      fence_mbarrier_init();
+    }
+    __syncwarp();
+    tmem_alloc<CG>(smem_u32(slot), 512);
+  }
+  tc_fence_before();
+  if constexpr (CG == 2) cluster_sync(); else __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *slot;
+  constexpr uint32_t IDESC = make_idesc_f16<M, N, false, false>();
+  if (warp == 0 && lane == 0 && rank == 0) {
+    const uint32_t sa = smem_u32(smem), sb = sa + 16384;
+    uint32_t phase = 0;
+    long long t0 = clock64();
+    if (!latency_mode) {
+      for (int i = 0; i < iters; ++i) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          umma_f16<CG>(tmem, sdesc_k_sw128(sa + 32 * k), sdesc_k_sw128(sb + 32 * k), IDESC, 1u);
+      }
+      umma_commit<CG>(bar);
+      mbar_wait(bar, 0);
+    } else {
+      for (int i = 0; i < iters; ++i) {
+        umma_f16<CG>(tmem, sdesc_k_sw128(sa), sdesc_k_sw128(sb), IDESC, 1u);
+        umma_commit<CG>(bar);
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+      }
+    }
+    long long t1 = clock64();
+    out[blockIdx.x] = static_cast<unsigned long long>(t1 - t0);
+  }
+  tc_fence_before();
+  if constexpr (CG == 2) cluster_sync(); else __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    tmem_dealloc<CG>(tmem, 512);
+  }
+#endif
+}
+
+// ------------------------------------------------------------------ TMEM load bandwidth
+__global__ void __launch_bounds__(256, 1) tmem_ld_kernel(int iters, int warps, int unroll, unsigned long long *out) {
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
+  __shared__ uint32_t slot;
+  const uint32_t warp = warp_id(), lane = lane_id();
+  if (warp == 0) tmem_alloc<1>(smem_u32(&slot), 512);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = slot;
+  unsigned long long sink = 0;
+  __syncthreads();
+  long long t0 = clock64();
+  if (warp < static_cast<uint32_t>(warps)) {
+    const uint32_t base = tmem + (((warp & 3u) * 32u) << 16) + (warp >> 2) * 256u;
+    if (unroll == 1) {
+      for (int i = 0; i < iters; ++i) {
+        uint32_t v[32];
+        tmem_ld_32x32b_x32(base + (i & 7) * 32, v);
+        tmem_ld_wait();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) sink += v[j];
+      }
+    } else {
+      for (int i = 0; i < iters; i += 4) {
+        uint32_t v0[32], v1[32], v2[32], v3[32];
+        tmem_ld_32x32b_x32(base + 0, v0);
+        tmem_ld_32x32b_x32(base + 32, v1);
+        tmem_ld_32x32b_x32(base + 64, v2);
+        tmem_ld_32x32b_x32(base + 96, v3);
+        tmem_ld_wait();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) sink += v0[j] + v1[j] + v2[j] + v3[j];
+      }
+    }
+  }
+  __syncthreads();
+  long long t1 = clock64();
+  if (threadIdx.x == 0) out[blockIdx.x] = static_cast<unsigned long long>(t1 - t0);
+  if (sink == 0x123456789ull) out[gridDim.x] = sink;
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    tmem_dealloc<1>(tmem, 512);
+  }
+#endif
+}
+
+// ------------------------------------------------------------------ TMA load bandwidth
+// One thread per CTA streams `iters` 128-row x 128-B boxes (16 KB) through a
+// ring of 8 stages.  stride_rows = 0 re-reads the same tile (L2 resident);
+// otherwise each CTA walks its own region of the tensor (HBM streaming).
+__global__ void __launch_bounds__(32, 1) tma_load_kernel(const __grid_constant__ CUtensorMap tm, int iters,
+                                                          int rows_total, int streaming, unsigned long long *out) {
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  uint8_t *smem = smem_raw + ((1024u - (raw & 1023u)) & 1023u);
+  uint64_t *full = reinterpret_cast<uint64_t *>(smem + 8 * 16384);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < 8; ++s) mbar_init(&full[s], 1);
+    fence_mbarrier_init();
+  }
+  __syncwarp();
+  if (threadIdx.x == 0) {
+    const int boxes_per_row = 8;  // 8 boxes of 64 FP16 across a 512-element row band
+    long long t0 = clock64();
+    uint32_t phase = 0;
+    for (int i = 0; i < iters + 8; ++i) {
+      const int s = i & 7;
+      if (i >= 8) {
+        mbar_wait(&full[s], phase);
+        if (s == 7) phase ^= 1u;
+      }
+      if (i < iters) {
+        int row = 0, col = 0;
+        if (streaming) {
+          const int64_t blk = static_cast<int64_t>(blockIdx.x) * iters + i;
+          col = static_cast<int>(blk % boxes_per_row) * 64;
+          row = static_cast<int>(((blk / boxes_per_row) * 128) % rows_total);
+        }
+        mbar_arrive_expect_tx(&full[s], 16384);
+        tma_load_2d(&tm, smem_u32(smem + s * 16384), smem_u32(&full[s]), col, row, 0);
+      }
+    }
+    long long t1 = clock64();
+    out[blockIdx.x] = static_cast<unsigned long long>(t1 - t0);
+  }
+#endif
+}
+
+}  // namespace mb
+
+namespace {
+using EncodeTiledFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                   const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  if (!fn) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &p, 12000, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  }
+  return fn;
+}
+}  // namespace
+
+extern "C" {
+
+// cycles[i] for CTA (or CTA pair) i; returns 0 on success.
+int mb_mma_rate(int cta_group, int n, int iters, int grid, int latency_mode, unsigned long long *cycles_dev) {
+  const int smem = 16384 + 256 * 128 + 1024 + 1024;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(128);
+  cfg.dynamicSmemBytes = smem;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = cta_group;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+#define MB_CASE(CG, NN)                                                                               \
+  if (cta_group == CG && n == NN) {                                                                   \
+    auto k = mb::mma_rate_kernel<CG, NN>;                                                             \
+    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                       \
+    return cudaLaunchKernelEx(&cfg, k, iters, cycles_dev, latency_mode) == cudaSuccess ? 0 : 1;       \
+  }
+  MB_CASE(1, 64)
+  MB_CASE(1, 128)
+  MB_CASE(1, 256)
+  MB_CASE(2, 64)
+  MB_CASE(2, 128)
+  MB_CASE(2, 256)
+#undef MB_CASE
+  return 2;
+}
+
+int mb_tmem_ld(int iters, int warps, int unroll, int grid, unsigned long long *cycles_dev) {
+  mb::tmem_ld_kernel<<<grid, 256>>>(iters, warps, unroll, cycles_dev);
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : 1;
+}
+
+// tensor: rows x 512 FP16 row-major device buffer (rows multiple of 128)
+int mb_tma_load(const void *tensor, int rows, int iters, int grid, int streaming, unsigned long long *cycles_dev) {
+  EncodeTiledFn fn = encode_fn();
+  if (!fn) return 3;
+  CUtensorMap tm;
+  cuuint64_t dims[2] = {512, static_cast<cuuint64_t>(rows)};
+  cuuint64_t strides[1] = {512 * 2};
+  cuuint32_t box[2] = {64, 128};
+  cuuint32_t estr[2] = {1, 1};
+  if (fn(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(tensor), dims, strides, box, estr,
+         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return 4;
+  const int smem = 8 * 16384 + 1024 + 1024;
+  cudaFuncSetAttribute(mb::tma_load_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  mb::tma_load_kernel<<<grid, 32, smem>>>(tm, iters, rows, streaming, cycles_dev);
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : 1;
+}
+
+}  // extern "C"
