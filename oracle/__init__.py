@@ -105,8 +105,9 @@ def hgemm_ref(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", transB="
         Cin = None
     size = ldc * n if n > 0 else 0
     C_out = np.zeros(max(size, 1), dtype=np.float32 if out_f32 else np.uint16)
-    if Cin is not None and Cin.size >= size:
-        C_out[:size] = Cin[:size]            # untouched padding rows keep their input bytes
+    if Cin is not None:
+        cnt = min(size, Cin.size)
+        C_out[:cnt] = Cin[:cnt]              # untouched padding rows keep their input bytes
     r = np.zeros((m, n), dtype=np.float64, order="F") if want_r else None
     ab = np.zeros((m, n), dtype=np.float64, order="F") if want_r else None
     rc = _load().hgemm_ref(m, n, k, float(alpha), _ptr(Ab), lda, _ptr(Bb), ldb, float(beta),

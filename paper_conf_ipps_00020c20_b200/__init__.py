@@ -9,4 +9,4 @@ The shared library is loaded on first use; a missing library raises.
 from .binding import (HGEMM_OUT_F16, HGEMM_OUT_F32, HgemmError, hgemm, hgemm_torch,  # noqa: F401
                       lib_path, load_library, status_string, set_config, get_stats,
                       set_probe, probe_clock_ghz)
-from .sharded import hgemm_sharded, slab_bounds  # noqa: F401
+from .sharded import hgemm_sharded, hgemm_sharded_overlapped, slab_bounds  # noqa: F401

@@ -84,6 +84,51 @@ def hgemm_sharded(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", tran
     return n0, n1
 
 
+def hgemm_sharded_overlapped(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="T", transB="N",
+                             out_dtype="f16", *, panels=4, group=None, src=0, local_slabs=False, gemm=None,
+                             stream=None):
+    """Sharded GEMM with the broadcast of A pipelined against the GEMM.
+
+    op(A) is split into `panels` row panels (m ranges).  With transA = 'T'
+    (A stored k x m, the paper's layout) row panel [m0, m1) of op(A) is the
+    contiguous column range A[:, m0:m1] = A + m0*lda, so each panel is one
+    contiguous NCCL broadcast.  All broadcasts are enqueued asynchronously
+    (in order on the communicator's stream); the GEMM of panel i
+    (C[m0:m1, slab] = op(A)[m0:m1, :] op(B)[:, slab], a pointer offset into C)
+    waits only for broadcast i, so it overlaps broadcasts i+1, i+2, ...
+    Every element is computed exactly as in the unpipelined path.
+    Returns this rank's (n0, n1)."""
+    import torch.distributed as dist
+    if transA not in ("T", "t"):
+        raise ValueError("row panels of op(A) are contiguous only for transA='T'")
+    world, rank = _world_rank(group)
+    n0, n1 = slab_bounds(n, world, rank)
+    if gemm is None:
+        from .binding import hgemm as gemm
+    f32 = str(out_dtype) in ("f32", "float32", "torch.float32", "1")
+    esz_c = 4 if f32 else 2
+    off_b, off_c = (0, 0) if local_slabs else slab_offsets(n0, ldb, ldc, transB, 2, esz_c)
+    bounds = [(m * i) // panels for i in range(panels + 1)]
+    bounds = [b - b % 8 if 0 < b < m else b for b in bounds]   # 16-B aligned panel starts
+    works = []
+    if world > 1:
+        flat = A.view(-1)
+        for i in range(panels):
+            p0, p1 = bounds[i], bounds[i + 1]
+            if p1 > p0:
+                works.append(dist.broadcast(flat[p0 * lda:p1 * lda], src=src, group=group, async_op=True))
+            else:
+                works.append(None)
+    for i in range(panels):
+        p0, p1 = bounds[i], bounds[i + 1]
+        if world > 1 and works[i] is not None:
+            works[i].wait()          # the compute stream waits for panel i only
+        if p1 > p0 and n1 > n0:
+            gemm(p1 - p0, n1 - n0, k, alpha, _offset(A, p0 * lda * 2), lda, _offset(B, off_b), ldb, beta,
+                 _offset(C, off_c + p0 * esz_c), ldc, transA, transB, out_dtype, stream)
+    return n0, n1
+
+
 class _Offset:
     """A (tensor, byte offset) pair that the binding's pointer marshalling accepts."""
 

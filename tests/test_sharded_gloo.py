@@ -14,7 +14,8 @@ import numpy as np
 import pytest
 
 from paper_conf_ipps_00020c20_b200 import inputs
-from paper_conf_ipps_00020c20_b200.sharded import hgemm_sharded, slab_bounds, slab_offsets
+from paper_conf_ipps_00020c20_b200.sharded import (hgemm_sharded, hgemm_sharded_overlapped, slab_bounds,
+                                                   slab_offsets)
 
 
 def test_slab_bounds_cover_and_align():
@@ -53,9 +54,10 @@ def _split(obj):
 def _oracle_gemm(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, tA, tB, out, stream):
     """Host stand-in for the CUDA hgemm with the same argument list (tests only)."""
     import oracle
+    At, aoff = _split(A)
     Bt, boff = _split(B)
     Ct, coff = _split(C)
-    a = A.numpy().view(np.uint16).reshape(-1)
+    a = At.numpy().view(np.uint16).reshape(-1)[aoff // 2:]
     b = Bt.numpy().view(np.uint16).reshape(-1)[boff // 2:]
     esz = 4 if out == "f32" else 2
     cflat = Ct.numpy().reshape(-1)
@@ -71,7 +73,8 @@ def _worker(rank, world, port, case, result_dir):
     import torch
     import torch.distributed as dist
     dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
-    m, n, k, tA, tB, alpha, beta, out, local = case
+    m, n, k, tA, tB, alpha, beta, out, local = case[:9]
+    overlap = len(case) > 9 and case[9]
     sa = inputs.stored_shape(m, k, tA)
     sb = inputs.stored_shape(k, n, tB)
     A_full = inputs.uniform_f16(sa[0], sa[1], 11)
@@ -98,8 +101,12 @@ def _worker(rank, world, port, case, result_dir):
     else:
         B = torch.from_numpy(B_full.reshape(-1, order="F").view(np.int16).copy())
         C = torch.from_numpy(C_full.reshape(-1, order="F").view(cv).copy())
-    got = hgemm_sharded(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, tA, tB, out,
-                        local_slabs=local, gemm=_oracle_gemm)
+    if overlap:
+        got = hgemm_sharded_overlapped(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, tA, tB, out, panels=3,
+                                       local_slabs=local, gemm=_oracle_gemm)
+    else:
+        got = hgemm_sharded(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, tA, tB, out,
+                            local_slabs=local, gemm=_oracle_gemm)
     assert got == (n0, n1)
     # A was replicated
     assert np.array_equal(A.numpy().view(np.uint16), A_full.reshape(-1, order="F").view(np.uint16))
@@ -115,12 +122,14 @@ def _worker(rank, world, port, case, result_dir):
     (37, 70, 45, "N", "T", 0.5, 1.0, "f32", False),
     (29, 53, 33, "T", "T", 1.0, -1.0, "f16", True),
     (16, 8, 64, "N", "N", 1.0, 0.0, "f32", True),
+    (41, 70, 45, "T", "N", 1.0, 0.5, "f16", False, True),     # NEXT-2: panel-pipelined broadcast
+    (64, 33, 80, "T", "T", -1.0, 0.0, "f32", True, True),
 ])
 def test_sharded_gloo_world2_bitwise(tmp_path, case, oracle_mod):
     import torch.multiprocessing as mp
     world = 2
     mp.spawn(_worker, args=(world, _free_port(), case, str(tmp_path)), nprocs=world, join=True)
-    m, n, k, tA, tB, alpha, beta, out, _ = case
+    m, n, k, tA, tB, alpha, beta, out = case[:8]
     slabs = [np.load(os.path.join(tmp_path, f"slab{r}.npy")) for r in range(world)]
     cat = np.concatenate(slabs, axis=1)
     # single-process reference on the same seeded inputs
