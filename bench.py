@@ -120,7 +120,8 @@ def max_over_ranks(x, world):
         return x
     import torch
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -214,11 +215,18 @@ def run_ours(args, world, rank, local):
     import torch
     from paper_conf_ipps_00020c20_b200 import binding, inputs
     from paper_conf_ipps_00020c20_b200.sharded import broadcast_A, hgemm_sharded, slab_bounds
+    # HGEMM_DIST_BACKEND=gloo lets several ranks share one GPU to exercise the N > 1
+    # code path where only one GPU is available (no performance meaning).
+    backend = os.environ.get("HGEMM_DIST_BACKEND", "nccl")
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     lib = binding.load_library()
     m, n_cfg, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[args.workload]
     strong = args.workload in inputs.STRONG_SCALING
@@ -262,9 +270,31 @@ def run_ours(args, world, rank, local):
         e1.record()
         torch.cuda.synchronize()
         bms = max_over_ranks(e0.elapsed_time(e1), world)
-        coll = {"op": "broadcast(A) over NCCL (torch.distributed)", "bytes": A.numel() * 2, "ms": bms,
+        coll = {"op": f"broadcast(A) over {dist.get_backend()} (torch.distributed)", "bytes": A.numel() * 2, "ms": bms,
                 "GB_s": A.numel() * 2 / (bms * 1e-3) / 1e9,
                 "note": "reported separately from the GEMM (north_star (3)); not inside value"}
+        # broadcast + GEMM as one step: serial, and pipelined in row panels of op(A) (NEXT-2)
+        if tA in ("T", "t"):
+            from paper_conf_ipps_00020c20_b200.sharded import hgemm_sharded_overlapped
+
+            def serial():
+                hgemm_sharded(m, n_glob, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out,
+                              broadcast=True, local_slabs=True, stream=stream.cuda_stream)
+
+            def overlapped():
+                hgemm_sharded_overlapped(m, n_glob, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out,
+                                         panels=args.panels, local_slabs=True, stream=stream.cuda_stream)
+            for name, fn in (("ms_bcast_then_gemm", serial), ("ms_bcast_gemm_pipelined", overlapped)):
+                fn()
+                torch.cuda.synchronize()
+                dist.barrier()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                fn()
+                e1.record()
+                torch.cuda.synchronize()
+                coll[name] = max_over_ranks(e0.elapsed_time(e1), world)
+            coll["pipeline_panels"] = args.panels
 
     def step():
         hgemm_sharded(m, n_glob, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out,
@@ -425,6 +455,7 @@ def main():
     ap.add_argument("--group-m", type=int, default=0)
     ap.add_argument("--ref-budget", type=float, default=60.0, help="seconds of oracle work for --impl reference")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
+    ap.add_argument("--panels", type=int, default=8, help="row panels of the pipelined broadcast (N > 1)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cublas", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
