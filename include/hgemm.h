@@ -72,6 +72,27 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k,
                      char transA, char transB, hgemm_dtype_t out_dtype,
                      cudaStream_t stream);
 
+/* Host-buffer variant: A, B and C are HOST pointers (page-locked memory gives
+ * full copy/compute overlap; pageable memory works but serialises the copies),
+ * same meaning, layout and quick-return rules as hgemm().  The call is
+ * SYNCHRONOUS: it returns after C has been written back to host memory.
+ * `workspace` is caller-owned DEVICE memory of at least
+ * hgemm_host_workspace_size(...) bytes (it holds the device copies of A, B
+ * and C).  The problem is processed in column panels of op(B)/C: panel j's
+ * host->device copy, GEMM and device->host copy run on three internal
+ * streams so the transfers of one panel overlap the GEMM of another.
+ * `stream` orders the whole call after prior work on it (0 = legacy stream).
+ * Errors: HGEMM_ERR_INVALID_VALUE as for hgemm(), also for a NULL or too
+ * small workspace; HGEMM_ERR_CUDA for copy/launch failures. */
+size_t hgemm_host_workspace_size(int64_t m, int64_t n, int64_t k, char transA, char transB,
+                                 hgemm_dtype_t out_dtype);
+hgemm_status_t hgemm_host(int64_t m, int64_t n, int64_t k,
+                          float alpha, const void *A, int64_t lda,
+                          const void *B, int64_t ldb,
+                          float beta, void *C, int64_t ldc,
+                          char transA, char transB, hgemm_dtype_t out_dtype,
+                          void *workspace, size_t workspace_bytes, cudaStream_t stream);
+
 /* Static, NUL-terminated description of a status code (never NULL). */
 const char *hgemm_status_string(hgemm_status_t s);
 

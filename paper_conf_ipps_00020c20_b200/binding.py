@@ -63,6 +63,11 @@ def load_library():
     lib.hgemm_set_config.restype = ctypes.c_int
     lib.hgemm_get_last_config.argtypes = [ctypes.POINTER(_Config)]
     lib.hgemm_get_last_config.restype = ctypes.c_int
+    lib.hgemm_host.argtypes = [i64, i64, i64, f32, vp, i64, vp, i64, f32, vp, i64,
+                               ctypes.c_char, ctypes.c_char, ctypes.c_int, vp, ctypes.c_size_t, vp]
+    lib.hgemm_host.restype = ctypes.c_int
+    lib.hgemm_host_workspace_size.argtypes = [i64, i64, i64, ctypes.c_char, ctypes.c_char, ctypes.c_int]
+    lib.hgemm_host_workspace_size.restype = ctypes.c_size_t
     lib.hgemm_set_probe.argtypes = [vp]
     lib.hgemm_set_probe.restype = ctypes.c_int
     lib.hgemm_launch_count.argtypes = []
@@ -149,6 +154,25 @@ def hgemm(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", transB="N",
     code = lib.hgemm(int(m), int(n), int(k), float(alpha), _ptr(A), int(lda), _ptr(B), int(ldb),
                      float(beta), _ptr(C), int(ldc), transA.encode()[:1], transB.encode()[:1],
                      _out_code(out_dtype), _stream(stream))
+    _check(code)
+
+
+def host_workspace_size(m, n, k, transA="N", transB="N", out_dtype=HGEMM_OUT_F16) -> int:
+    return int(load_library().hgemm_host_workspace_size(int(m), int(n), int(k), transA.encode()[:1],
+                                                        transB.encode()[:1], _out_code(out_dtype)))
+
+
+def hgemm_host(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", transB="N",
+               out_dtype=HGEMM_OUT_F16, workspace=None, workspace_bytes=None, stream=None):
+    """Host-buffer variant (include/hgemm.h): A, B, C are HOST pointers / CPU tensors
+    (pinned for copy-compute overlap); `workspace` is device memory of at least
+    host_workspace_size(...) bytes.  Synchronous."""
+    lib = load_library()
+    if workspace_bytes is None:
+        workspace_bytes = int(workspace.numel() * workspace.element_size()) if workspace is not None else 0
+    code = lib.hgemm_host(int(m), int(n), int(k), float(alpha), _ptr(A), int(lda), _ptr(B), int(ldb), float(beta),
+                          _ptr(C), int(ldc), transA.encode()[:1], transB.encode()[:1], _out_code(out_dtype),
+                          _ptr(workspace), int(workspace_bytes), _stream(stream))
     _check(code)
 
 

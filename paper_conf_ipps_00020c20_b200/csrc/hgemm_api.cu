@@ -84,9 +84,42 @@ EncodeTiledFn encode_fn() {
 
 // 2-D tensor with 128-B swizzled boxes: `inner` contiguous elements per line,
 // `outer` lines `ld` elements apart.  FP16 operands (loads) or the FP16/FP32
-// output D (epilogue stores).
+// output D (epilogue stores).  Encoded maps are cached (keyed by every encode
+// argument): repeated calls on the same buffers skip cuTensorMapEncodeTiled.
+// A cached map is a plain value copied into the launch parameters; nothing is
+// dereferenced on the host.
+struct MapKey {
+  const void *base;
+  uint64_t inner, outer;
+  int64_t ld;
+  uint32_t box_inner, box_outer;
+  int f32;
+  bool operator==(const MapKey &o) const {
+    return base == o.base && inner == o.inner && outer == o.outer && ld == o.ld && box_inner == o.box_inner &&
+           box_outer == o.box_outer && f32 == o.f32;
+  }
+};
+constexpr int kMapCache = 32;
+struct MapCache {
+  MapKey key[kMapCache];
+  CUtensorMap map[kMapCache];
+  bool valid[kMapCache] = {};
+  int next = 0;
+  std::mutex mu;
+};
+MapCache g_maps;
+
 bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer, int64_t ld, uint32_t box_inner,
               uint32_t box_outer, bool f32 = false) {
+  const MapKey key = {base, inner, outer, ld, box_inner, box_outer, f32 ? 1 : 0};
+  {
+    std::lock_guard<std::mutex> lk(g_maps.mu);
+    for (int i = 0; i < kMapCache; ++i)
+      if (g_maps.valid[i] && g_maps.key[i] == key) {
+        *map = g_maps.map[i];
+        return true;
+      }
+  }
   EncodeTiledFn fn = encode_fn();
   if (!fn) return false;
   const int esz = f32 ? 4 : 2;
@@ -97,7 +130,14 @@ bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer
   CUresult r = fn(map, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2,
                   const_cast<void *>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  return r == CUDA_SUCCESS;
+  if (r != CUDA_SUCCESS) return false;
+  std::lock_guard<std::mutex> lk(g_maps.mu);
+  const int slot = g_maps.next;
+  g_maps.next = (g_maps.next + 1) % kMapCache;
+  g_maps.key[slot] = key;
+  g_maps.map[slot] = *map;
+  g_maps.valid[slot] = true;
+  return true;
 }
 
 // ----------------------------------------------------------------- TC launch
@@ -501,6 +541,148 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0};
   }
   return st;
+}
+
+}  // extern "C"
+
+// ===================================================================== host-buffer path
+namespace {
+
+struct HostPipe {
+  bool init = false;
+  cudaStream_t s_in = nullptr, s_comp = nullptr, s_out = nullptr;
+  static constexpr int kEv = 64;
+  cudaEvent_t ev_in[kEv] = {}, ev_comp[kEv] = {}, ev_start = nullptr;
+};
+HostPipe g_pipe[kMaxDevices];
+std::mutex g_pipe_mu;
+
+inline int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+
+struct HostLayout {
+  int64_t a_rows, a_cols, b_rows, b_cols;  // stored shapes
+  int64_t off_a, off_b, off_c, total;      // workspace offsets (bytes)
+};
+
+HostLayout host_layout(int64_t m, int64_t n, int64_t k, bool tA, bool tB, bool f32) {
+  HostLayout L;
+  L.a_rows = tA ? k : m;
+  L.a_cols = tA ? m : k;
+  L.b_rows = tB ? n : k;
+  L.b_cols = tB ? k : n;
+  // device copies keep a 16-byte aligned pitch (the TMA fast-path precondition)
+  const int64_t lda_d = align_up(std::max<int64_t>(L.a_rows, 1), 8);
+  const int64_t ldb_d = align_up(std::max<int64_t>(L.b_rows, 1), 8);
+  const int64_t ldc_d = align_up(std::max<int64_t>(m, 1), f32 ? 4 : 8);
+  L.off_a = 0;
+  L.off_b = align_up(L.off_a + lda_d * L.a_cols * 2, 256);
+  L.off_c = align_up(L.off_b + ldb_d * L.b_cols * 2, 256);
+  L.total = align_up(L.off_c + ldc_d * n * (f32 ? 4 : 2), 256);
+  return L;
+}
+
+}  // namespace
+
+extern "C" {
+
+size_t hgemm_host_workspace_size(int64_t m, int64_t n, int64_t k, char transA, char transB,
+                                 hgemm_dtype_t out_dtype) {
+  if (m < 0 || n < 0 || k < 0) return 0;
+  return static_cast<size_t>(host_layout(m, n, k, is_t(transA), is_t(transB), out_dtype == HGEMM_OUT_F32).total);
+}
+
+hgemm_status_t hgemm_host(int64_t m, int64_t n, int64_t k, float alpha, const void *A, int64_t lda, const void *B,
+                          int64_t ldb, float beta, void *C, int64_t ldc, char transA, char transB,
+                          hgemm_dtype_t out_dtype, void *workspace, size_t workspace_bytes, cudaStream_t stream) {
+  if (m < 0 || n < 0 || k < 0) return HGEMM_ERR_INVALID_VALUE;
+  if (!(is_t(transA) || is_n(transA)) || !(is_t(transB) || is_n(transB))) return HGEMM_ERR_INVALID_VALUE;
+  if (out_dtype != HGEMM_OUT_F16 && out_dtype != HGEMM_OUT_F32) return HGEMM_ERR_INVALID_VALUE;
+  const bool tA = is_t(transA), tB = is_t(transB), f32 = (out_dtype == HGEMM_OUT_F32);
+  if (lda < std::max<int64_t>(1, tA ? k : m)) return HGEMM_ERR_INVALID_VALUE;
+  if (ldb < std::max<int64_t>(1, tB ? n : k)) return HGEMM_ERR_INVALID_VALUE;
+  if (ldc < std::max<int64_t>(1, m)) return HGEMM_ERR_INVALID_VALUE;
+  if (m == 0 || n == 0) return HGEMM_SUCCESS;
+  if (!C) return HGEMM_ERR_INVALID_VALUE;
+  const bool need_ab = (k > 0 && alpha != 0.0f);
+  if (need_ab && (!A || !B)) return HGEMM_ERR_INVALID_VALUE;
+  const HostLayout L = host_layout(m, n, k, tA, tB, f32);
+  if (!workspace || workspace_bytes < static_cast<size_t>(L.total)) return HGEMM_ERR_INVALID_VALUE;
+
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return HGEMM_ERR_CUDA;
+  HostPipe &P = g_pipe[dev];
+  {
+    std::lock_guard<std::mutex> lk(g_pipe_mu);
+    if (!P.init) {
+      if (cudaStreamCreateWithFlags(&P.s_in, cudaStreamNonBlocking) != cudaSuccess ||
+          cudaStreamCreateWithFlags(&P.s_comp, cudaStreamNonBlocking) != cudaSuccess ||
+          cudaStreamCreateWithFlags(&P.s_out, cudaStreamNonBlocking) != cudaSuccess ||
+          cudaEventCreateWithFlags(&P.ev_start, cudaEventDisableTiming) != cudaSuccess)
+        return HGEMM_ERR_CUDA;
+      for (int i = 0; i < HostPipe::kEv; ++i)
+        if (cudaEventCreateWithFlags(&P.ev_in[i], cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&P.ev_comp[i], cudaEventDisableTiming) != cudaSuccess)
+          return HGEMM_ERR_CUDA;
+      P.init = true;
+    }
+  }
+  std::lock_guard<std::mutex> call_lk(g_pipe_mu);  // the pipeline streams/events serve one call at a time
+  const int esz = f32 ? 4 : 2;
+  uint8_t *ws = static_cast<uint8_t *>(workspace);
+  const int64_t lda_d = align_up(std::max<int64_t>(L.a_rows, 1), 8);
+  const int64_t ldb_d = align_up(std::max<int64_t>(L.b_rows, 1), 8);
+  const int64_t ldc_d = align_up(std::max<int64_t>(m, 1), f32 ? 4 : 8);
+  void *dA = ws + L.off_a, *dB = ws + L.off_b, *dC = ws + L.off_c;
+
+  // panel width: >= 1024 columns, at most kEv panels, a multiple of 256
+  int64_t panels = std::min<int64_t>(HostPipe::kEv - 1, std::max<int64_t>(1, n / 1024));
+  if (panels > 8) panels = 8;
+  int64_t pw = align_up(cdiv(n, panels), 256);
+  panels = cdiv(n, pw);
+
+  if (cudaEventRecord(P.ev_start, stream) != cudaSuccess) return HGEMM_ERR_CUDA;
+  if (cudaStreamWaitEvent(P.s_in, P.ev_start, 0) != cudaSuccess) return HGEMM_ERR_CUDA;
+  if (need_ab) {
+    if (cudaMemcpy2DAsync(dA, lda_d * 2, A, lda * 2, L.a_rows * 2, L.a_cols, cudaMemcpyHostToDevice, P.s_in) !=
+        cudaSuccess)
+      return HGEMM_ERR_CUDA;
+  }
+  for (int64_t j = 0; j < panels; ++j) {
+    const int64_t n0 = j * pw, n1 = std::min(n, n0 + pw), w = n1 - n0;
+    if (need_ab) {
+      // op(B)[:, n0:n1]: B columns (transB 'N') or B rows (transB 'T')
+      const uint8_t *src = static_cast<const uint8_t *>(B) + (tB ? n0 : n0 * ldb) * 2;
+      uint8_t *dst = static_cast<uint8_t *>(dB) + (tB ? n0 : n0 * ldb_d) * 2;
+      const size_t width = static_cast<size_t>(tB ? w : L.b_rows) * 2;
+      const size_t height = static_cast<size_t>(tB ? L.b_cols : w);
+      if (cudaMemcpy2DAsync(dst, ldb_d * 2, src, ldb * 2, width, height, cudaMemcpyHostToDevice, P.s_in) !=
+          cudaSuccess)
+        return HGEMM_ERR_CUDA;
+    }
+    if (beta != 0.0f) {
+      if (cudaMemcpy2DAsync(static_cast<uint8_t *>(dC) + n0 * ldc_d * esz, ldc_d * esz,
+                            static_cast<const uint8_t *>(C) + n0 * ldc * esz, ldc * esz, m * esz, w,
+                            cudaMemcpyHostToDevice, P.s_in) != cudaSuccess)
+        return HGEMM_ERR_CUDA;
+    }
+    if (cudaEventRecord(P.ev_in[j], P.s_in) != cudaSuccess) return HGEMM_ERR_CUDA;
+    if (cudaStreamWaitEvent(P.s_comp, P.ev_in[j], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
+    const void *dBj = static_cast<const uint8_t *>(dB) + (tB ? n0 : n0 * ldb_d) * 2;
+    void *dCj = static_cast<uint8_t *>(dC) + n0 * ldc_d * esz;
+    const hgemm_status_t st = hgemm(m, w, k, alpha, dA, lda_d, dBj, ldb_d, beta, dCj, ldc_d, transA, transB,
+                                    out_dtype, P.s_comp);
+    if (st != HGEMM_SUCCESS) return st;
+    if (cudaEventRecord(P.ev_comp[j], P.s_comp) != cudaSuccess) return HGEMM_ERR_CUDA;
+    if (cudaStreamWaitEvent(P.s_out, P.ev_comp[j], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
+    if (cudaMemcpy2DAsync(static_cast<uint8_t *>(C) + n0 * ldc * esz, ldc * esz, dCj, ldc_d * esz, m * esz, w,
+                          cudaMemcpyDeviceToHost, P.s_out) != cudaSuccess)
+      return HGEMM_ERR_CUDA;
+  }
+  // make `stream` observe the end of the pipeline (events recorded on it bracket the whole call)
+  if (cudaEventRecord(P.ev_comp[HostPipe::kEv - 1], P.s_out) != cudaSuccess) return HGEMM_ERR_CUDA;
+  if (cudaStreamWaitEvent(stream, P.ev_comp[HostPipe::kEv - 1], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
+  if (cudaStreamSynchronize(P.s_out) != cudaSuccess) return HGEMM_ERR_CUDA;
+  return HGEMM_SUCCESS;
 }
 
 }  // extern "C"

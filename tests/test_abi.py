@@ -76,3 +76,18 @@ def test_kernel_sass_is_blackwell_native():
     assert "UTCHMMA" in sass and "UTMALDG" in sass and "LDTM" in sass
     assert "UTCHMMA.2CTA" in sass
     assert " HMMA" not in sass
+
+
+def test_host_entry_validation():
+    lib = binding.load_library()
+    need = binding.host_workspace_size(100, 200, 300, "T", "N", "f16")
+    # A (300 x 100 -> pitch 304), B (300 x 200 -> 304), C (100 x 200 -> 104), 256-byte aligned segments
+    up = lambda x: (x + 255) // 256 * 256
+    assert need == up(304 * 100 * 2) + up(304 * 200 * 2) + up(104 * 200 * 2)
+    assert binding.host_workspace_size(-1, 2, 3, "N", "N", "f16") == 0
+    # too small a workspace is an argument error (checked before any CUDA call)
+    assert lib.hgemm_host(100, 200, 300, 1.0, 16, 300, 16, 300, 0.0, 16, 100, b"T", b"N", 0, 16, need - 1,
+                          None) == 1
+    assert lib.hgemm_host(100, 200, 300, 1.0, 16, 300, 16, 300, 0.0, 16, 100, b"T", b"N", 0, None, need,
+                          None) == 1
+    assert lib.hgemm_host(100, 200, 300, 1.0, 16, 10, 16, 300, 0.0, 16, 100, b"T", b"N", 0, 16, need, None) == 1

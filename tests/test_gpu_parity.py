@@ -241,3 +241,51 @@ def test_splitk_auto_for_underfilled(oracle_mod):
     assert case.stats["last_kernel"] == "splitk", case.stats
     _, r, ab = case.oracle(oracle_mod)
     assert_within_tolerance(case, got, r, ab)
+
+
+def test_cuda_graph_capture_and_replay(oracle_mod):
+    """hgemm() is asynchronous and allocation-free, so it can be captured in a CUDA graph."""
+    import torch
+    from paper_conf_ipps_00020c20_b200 import binding
+    m, n, k = 384, 640, 512
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", 1.0, 0.0, out="f32")
+    dA = torch.from_numpy(case.A.view(np.int16).copy()).cuda()
+    dB = torch.from_numpy(case.B.view(np.int16).copy()).cuda()
+    dC = torch.full((case.ldc * n,), float("nan"), dtype=torch.float32, device="cuda")
+    g = torch.cuda.CUDAGraph()
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        with torch.cuda.graph(g, stream=s):
+            binding.hgemm(m, n, k, 1.0, dA, case.lda, dB, case.ldb, 0.0, dC, case.ldc, "T", "N", "f32",
+                          s.cuda_stream)
+    dC.fill_(float("nan"))
+    g.replay()
+    torch.cuda.synchronize()
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, dC.cpu().numpy(), r, ab)
+
+
+@pytest.mark.parametrize("tA,tB", TRANS)
+@pytest.mark.parametrize("out,beta", [("f16", 0.0), ("f16", 1.0), ("f32", 0.5)])
+def test_hgemm_host_buffers(oracle_mod, tA, tB, out, beta):
+    """Host-buffer entry point: panelled H2D / GEMM / D2H pipeline gives the same C."""
+    import torch
+    from paper_conf_ipps_00020c20_b200 import binding
+    m, n, k = 300, 2600, 520            # several column panels + ragged tails; host ld padding
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), tA, tB, 1.0, beta,
+                   C=inputs.uniform_f16(m, n, 3), out=out, pad=(3, 5, 7), align=False)
+    hA = torch.from_numpy(case.A.view(np.int16).copy()).pin_memory()
+    hB = torch.from_numpy(case.B.view(np.int16).copy()).pin_memory()
+    cv = case.C_in.view(np.int16) if out == "f16" else case.C_in
+    hC = torch.from_numpy(cv.copy()).pin_memory()
+    ws_bytes = binding.host_workspace_size(m, n, k, tA, tB, out)
+    ws = torch.empty(ws_bytes, dtype=torch.uint8, device="cuda")
+    binding.hgemm_host(m, n, k, 1.0, hA, case.lda, hB, case.ldb, beta, hC, case.ldc, tA, tB, out, ws)
+    got = hC.numpy()
+    if out == "f16":
+        got = got.view(np.float16)
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, got, r, ab)
+    # the host padding rows of C are untouched
+    pad = case.padding(got).astype(np.float32)
+    assert np.all(np.isnan(pad))
