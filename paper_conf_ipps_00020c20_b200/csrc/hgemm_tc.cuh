@@ -246,6 +246,11 @@ __device__ __forceinline__ void load_c_words(const TcParams &p, uint32_t (&cw)[C
   }
 }
 
+// k-blocks by which accumulator half 1 trails half 0 at the end of a 512-wide tile
+#ifndef HGEMM_END_LAG
+#define HGEMM_END_LAG 2
+#endif
+
 // HGEMM_TRACE (experiments only): CTA 0 records clock64 timestamps of the
 // accumulator hand-off into p.probe[8 + 8*tile + field] for its first 16 tiles.
 #ifdef HGEMM_TRACE
@@ -290,8 +295,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
   uint8_t *epi_smem = smem + STAGES * STAGE_BYTES;
   uint64_t *full = reinterpret_cast<uint64_t *>(epi_smem + S::EPI_BYTES);
   uint64_t *empty = full + STAGES;
-  uint64_t *tfull = empty + STAGES;      // [ACC]
-  uint64_t *tempty = tfull + ACC;        // [ACC][NH]
+  uint64_t *tfull = empty + STAGES;      // [ACC][NH]
+  uint64_t *tempty = tfull + ACC * NH;   // [ACC][NH]
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + ACC * NH);
 
   const uint32_t warp = warp_id();
@@ -313,8 +318,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         mbar_init(&empty[s], 1);
       }
       for (int a = 0; a < ACC; ++a) {
-        mbar_init(&tfull[a], 1);
-        for (int h = 0; h < NH; ++h) mbar_init(&tempty[a * NH + h], S::EPI_WARPS * CG);
+        for (int h = 0; h < NH; ++h) {
+          mbar_init(&tfull[a * NH + h], 1);
+          mbar_init(&tempty[a * NH + h], S::EPI_WARPS * CG);
+        }
       }
       fence_mbarrier_init();
     }
@@ -389,23 +396,66 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (leader CTA)
     if (rank == 0 && lane == 0) {
-      // For NH == 2 the second accumulator half may still be draining when a
-      // tile starts: half-0 MMAs then run up to MAX_LEAD k-blocks ahead (their
-      // smem stages stay resident) until tempty[half 1] is acquired.
+      // NH == 2 (one 512-column accumulator in two halves):
+      //  * at a tile start, half 1 may still be draining: half-0 MMAs run up to
+      //    MAX_LEAD k-blocks ahead (their smem stages stay resident) until
+      //    tempty[half 1] is acquired;
+      //  * at a tile end, half 1 deliberately lags half 0 by END_LAG k-blocks and
+      //    each half has its own tmem_full barrier, so the epilogue drains half 0
+      //    while the tensor core finishes half 1 and the next tile's half 0 can
+      //    start as soon as the previous half 0 is drained;
+      //  * in between, the halves are interleaved per K step (consecutive MMAs
+      //    share the A descriptor).
       constexpr int MAX_LEAD = STAGES - 1;
       uint32_t stage = 0, phase = 0;
       int it = 0;
+      auto issue_half = [&](uint32_t st, int h, int kbl, uint32_t d_tmem) {
+        const uint32_t sa = smem_u32(smem + st * STAGE_BYTES);
+#pragma unroll
+        for (int k = 0; k < BK / 16; ++k) {
+          const uint32_t a_addr = sa + k * A_KSTEP;
+          const uint32_t b_addr = sa + A_BYTES + h * B_HALF_BYTES + k * B_KSTEP;
+          const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+          const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
+          umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kbl | k) != 0 ? 1u : 0u);
+        }
+      };
+      const int nkb = p.num_k_blocks;
+      const int end_lag = (NH == 2) ? min(HGEMM_END_LAG, max(nkb - 1, 0)) : 0;
+      const int h1_limit = nkb - end_lag;  // half-1 k-blocks >= h1_limit are issued after the loop
       for (int t = cluster_id; t < num_tiles; t += num_clusters, ++it) {
         const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
         const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
         const uint32_t d_tmem = tmem_base + buf * BN;
         bool h1_ready = (NH == 1);
-        int pend_lo = 0;              // first k-block whose half-1 MMAs are not issued yet
-        uint32_t pend_stage = stage;  // its ring stage
+        int kb1 = 0;              // next k-block whose half-1 MMAs are not issued yet
+        uint32_t stage1 = stage;  // its ring stage
+        auto acquire_h1 = [&](bool block) {
+          if (block) {
+            if constexpr (CG == 2) mbar_wait_cluster(&tempty[buf * NH + 1], acc_phase ^ 1u);
+            else mbar_wait(&tempty[buf * NH + 1], acc_phase ^ 1u);
+            h1_ready = true;
+          } else {
+            const uint32_t te = smem_u32(&tempty[buf * NH + 1]);
+            h1_ready = (CG == 2) ? mbar_try_wait_cluster(te, acc_phase ^ 1u) : mbar_try_wait(te, acc_phase ^ 1u);
+          }
+          if (h1_ready) {
+            tc_fence_after();
+            HG_TRACE(it, 5);
+          }
+        };
+        auto flush_h1 = [&](int upto) {  // issue half 1 for k-blocks [kb1, upto)
+          while (kb1 < upto) {
+            issue_half(stage1, 1, kb1, d_tmem);
+            umma_commit<CG>(&empty[stage1]);  // both halves have consumed this stage
+            if (++stage1 == STAGES) stage1 = 0;
+            ++kb1;
+          }
+        };
 #ifdef HGEMM_TRACE
         long long full_wait = 0;
 #endif
-        for (int kb = 0; kb < p.num_k_blocks; ++kb) {
+        for (int kb = 0; kb < nkb; ++kb) {
 #ifdef HGEMM_TRACE
           const long long tw0 = clock64();
 #endif
@@ -422,74 +472,42 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
             tc_fence_after();
             HG_TRACE(it, 4);
           }
-          const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
-          // Steady state: interleave the halves per K step (consecutive MMAs share
-          // the A descriptor).
-          if (NH == 2 && h1_ready && pend_lo == kb) {
-#pragma unroll
-            for (int k = 0; k < BK / 16; ++k) {
-              const uint32_t a_addr = sa + k * A_KSTEP;
-              const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
-#pragma unroll
-              for (int h = 0; h < NH; ++h) {
-                const uint32_t b_addr = sa + A_BYTES + h * B_HALF_BYTES + k * B_KSTEP;
-                const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
-                umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
-              }
-            }
-            umma_commit<CG>(&empty[stage]);
-            pend_lo = kb + 1;
-            if (++pend_stage == STAGES) pend_stage = 0;
-            if (++stage == STAGES) { stage = 0; phase ^= 1u; }
-            continue;
-          }
-#pragma unroll
-          for (int k = 0; k < BK / 16; ++k) {
-            const uint32_t a_addr = sa + k * A_KSTEP;
-            const uint32_t b_addr = sa + A_BYTES + k * B_KSTEP;
-            const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
-            const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
-            umma_f16<CG>(d_tmem, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
-          }
           if constexpr (NH == 2) {
-            if (!h1_ready) {
-              const uint32_t te = smem_u32(&tempty[buf * NH + 1]);
-              if (kb - pend_lo + 1 >= MAX_LEAD || kb == p.num_k_blocks - 1) {
-                if constexpr (CG == 2) mbar_wait_cluster(&tempty[buf * NH + 1], acc_phase ^ 1u);
-                else mbar_wait(&tempty[buf * NH + 1], acc_phase ^ 1u);
-                h1_ready = true;
-              } else {
-                h1_ready = (CG == 2) ? mbar_try_wait_cluster(te, acc_phase ^ 1u) : mbar_try_wait(te, acc_phase ^ 1u);
-              }
-              if (h1_ready) {
-                tc_fence_after();
-                HG_TRACE(it, 5);
-              }
-            }
-            if (h1_ready) {
-              uint32_t s2 = pend_stage;
-              for (int j = pend_lo; j <= kb; ++j) {
-                const uint32_t sa2 = smem_u32(smem + s2 * STAGE_BYTES);
+            if (h1_ready && kb1 == kb && kb < h1_limit) {
+              const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
 #pragma unroll
-                for (int k = 0; k < BK / 16; ++k) {
-                  const uint32_t a_addr = sa2 + k * A_KSTEP;
-                  const uint32_t b_addr = sa2 + A_BYTES + B_HALF_BYTES + k * B_KSTEP;
-                  const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+              for (int k = 0; k < BK / 16; ++k) {
+                const uint32_t a_addr = sa + k * A_KSTEP;
+                const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+#pragma unroll
+                for (int h = 0; h < NH; ++h) {
+                  const uint32_t b_addr = sa + A_BYTES + h * B_HALF_BYTES + k * B_KSTEP;
                   const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
-                  umma_f16<CG>(d_tmem + UMMA_N, ad, bd, IDESC, (j | k) != 0 ? 1u : 0u);
+                  umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
                 }
-                umma_commit<CG>(&empty[s2]);  // both halves have consumed this stage
-                if (++s2 == STAGES) s2 = 0;
               }
-              pend_lo = kb + 1;
-              pend_stage = s2;
+              umma_commit<CG>(&empty[stage]);
+              ++kb1;
+              if (++stage1 == STAGES) stage1 = 0;
+            } else {
+              issue_half(stage, 0, kb, d_tmem);
+              if (!h1_ready) acquire_h1(kb - kb1 + 1 >= MAX_LEAD || kb == nkb - 1);
+              if (h1_ready) flush_h1(min(kb + 1, h1_limit));
             }
           } else {
+            issue_half(stage, 0, kb, d_tmem);
             umma_commit<CG>(&empty[stage]);  // frees the smem stage once these MMAs retire
           }
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
         }
-        umma_commit<CG>(&tfull[buf]);      // accumulator ready for the epilogue
+        if constexpr (NH == 2) {
+          umma_commit<CG>(&tfull[buf * NH + 0]);  // half 0 complete: the epilogue may drain it
+          if (!h1_ready) acquire_h1(true);
+          flush_h1(nkb);                            // the lagging half-1 k-blocks
+          umma_commit<CG>(&tfull[buf * NH + 1]);
+        } else {
+          umma_commit<CG>(&tfull[buf]);             // accumulator ready for the epilogue
+        }
         HG_TRACE(it, 0);
 #ifdef HGEMM_TRACE
         if (p.probe != nullptr && blockIdx.x == 0 && it < 16) p.probe[8 + 16 * it + 7] = full_wait;
@@ -530,7 +548,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       // One thread polls the accumulator barrier; the other epilogue warps
       // sleep on a named barrier instead of spinning.
       if (warp == 2 && lane == 0) {
-        mbar_wait(&tfull[buf], acc_phase);
+        mbar_wait(&tfull[buf * NH], acc_phase);
         HG_TRACE(it, 1);
       }
       named_bar_sync(1, 32 * S::EPI_WARPS);
@@ -543,6 +561,11 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         // back to the MMA warp, then store.
 #pragma unroll 1
         for (int h = 0; h < NH; ++h) {
+          if (h > 0) {  // each half has its own tmem_full barrier
+            if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
+            __syncwarp();
+            tc_fence_after();
+          }
           uint32_t pk[PKW];
           const int c0 = h * UMMA_N + cgrp * EPI_COLS_W;  // first tile column of this warp
           if (!pre_c) {
@@ -607,6 +630,11 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       }
 #pragma unroll 1
       for (int h = 0; h < NH; ++h) {
+        if (h > 0) {
+          if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
+          __syncwarp();
+          tc_fence_after();
+        }
 #pragma unroll 1
         for (int c = 0; c < EPI_COLS_W / EPI_COLS; ++c) {
           // column within the tile (= TMEM column offset)
