@@ -543,7 +543,17 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       uint32_t cw[OUT_F32 ? 1 : EPI_COLS_W / 2];
       const bool pre_c = !OUT_F32 && fast && beta != 0.0f;
       if constexpr (!OUT_F32) {
-        if (pre_c) load_c_words<EPI_COLS_W>(p, cw, row, tn * BN + cgrp * EPI_COLS_W);
+        if (pre_c) {
+          load_c_words<EPI_COLS_W>(p, cw, row, tn * BN + cgrp * EPI_COLS_W);
+          // half 1's C is loaded only after half 0 is stored: pull it into L2 now
+          if (NH > 1 && row < p.M) {
+            const __half *c1 = static_cast<const __half *>(p.D) + static_cast<int64_t>(row) * p.ldd + tn * BN +
+                               UMMA_N + cgrp * EPI_COLS_W;
+#pragma unroll
+            for (int q = 0; q < EPI_COLS_W * 2 / 128; ++q)
+              if (tn * BN + UMMA_N + cgrp * EPI_COLS_W + q * 64 < p.N) prefetch_l2(c1 + q * 64);
+          }
+        }
       }
       // One thread polls the accumulator barrier; the other epilogue warps
       // sleep on a named barrier instead of spinning.
