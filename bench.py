@@ -384,9 +384,16 @@ def run_ours(args, world, rank, local):
             opB = Bs.t() if tB in ("N", "n") else Bs
             X, Y = opB.t(), opA.t()
 
+            # same alpha/beta semantics: beta != 0 reads and rewrites C in place (addmm)
+            Cc = C.clone() if beta != 0 else None
+
             def cub():
+                if beta != 0:
+                    if out_t == torch.float16:
+                        return torch.addmm(Cc, X, Y, beta=beta, alpha=alpha, out=Cc)
+                    return torch.addmm(Cc, X, Y, out_dtype=torch.float32, beta=beta, alpha=alpha, out=Cc)
                 if out_t == torch.float16:
-                    return torch.mm(X, Y)
+                    return torch.mm(X, Y) if alpha == 1 else torch.mm(X, Y).mul_(alpha)
                 return torch.mm(X, Y, out_dtype=torch.float32)
             ref_c = cub()
             for _ in range(3):
@@ -405,7 +412,8 @@ def run_ours(args, world, rank, local):
             diff = (ref_c.float() - C.float()).abs().max().item() if beta == 0 else None
             cms = statistics.mean(a.elapsed_time(b) for a, b in ts)
             cublas = {"value": flops_rank / (cms * 1e-3) / 1e12, "unit": UNIT, "ms": cms, "max_abs_diff_vs_ours": diff,
-                      "what": "torch.mm (cuBLAS), same operands and layout, fp16 reduced-precision reduction off"}
+                      "what": ("torch.addmm(C, ..., beta, alpha, out=C)" if beta != 0 else "torch.mm") +
+                              " (cuBLAS), same operands, layout and alpha/beta, fp16 reduced-precision reduction off"}
         except Exception as e:  # pragma: no cover
             cublas = {"error": f"{type(e).__name__}: {e}"}
 

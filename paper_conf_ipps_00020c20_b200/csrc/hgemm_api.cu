@@ -140,10 +140,75 @@ bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer
   return true;
 }
 
+// ----------------------------------------------------------------- stream-K
+// Stream-K plan for `tiles` tiles of `nkb` k-blocks on `units` persistent
+// clusters: whole waves minus one run data-parallel, the rest is split into
+// one contiguous k range per cluster.  mode: 0 auto, 1 never, 2 always.
+// Returns the number of data-parallel tiles, or -1 for "no stream-K".
+// Every cluster range must hold >= 2 k-blocks (each partial slot is then
+// written at most once per launch).
+// Cost of stream-K in waves, measured (tools/tile_choice.py): the
+// 256-wide tiles are L2-throughput bound, so spreading the same L2 traffic over
+// more SMs gains nothing by itself; the FP32 fixup traffic and the lost
+// lockstep between clusters sharing panels cost about a third of a wave.  Stream-K
+// pays off only when the last data-parallel wave is nearly empty.
+inline double sk_overhead_waves(int64_t nkb) { return 0.35 + 4.0 / static_cast<double>(nkb); }
+int sk_plan(int64_t tiles, int64_t units, int64_t nkb, int mode) {
+  if (mode == 1 || units <= 1 || tiles % units == 0 || nkb < 2) return -1;
+  const int64_t dp = tiles > units ? (tiles / units - 1) * units : 0;
+  if ((tiles - dp) * nkb < 2 * units) return -1;
+  if (mode == 0) {
+    const double waves_dp = static_cast<double>((tiles + units - 1) / units);
+    const double waves_sk = static_cast<double>(tiles) / units + sk_overhead_waves(nkb);
+    if (nkb < 8 || waves_sk >= waves_dp) return -1;
+  }
+  return static_cast<int>(dp);
+}
+
+// Library-owned FP32 partial slots + flags, one set per (device, stream):
+// room for one 128 x 256 FP32 slot and one flag per SM.  Flags are zero
+// between launches (every consumer resets the flag it waited for).
+struct SkWorkspace {
+  int dev;
+  cudaStream_t stream;
+  float *ws;
+  int *flags;
+};
+std::mutex g_skws_mu;
+SkWorkspace g_skws[256];
+int g_skws_n = 0;
+
+bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags) {
+  std::lock_guard<std::mutex> lk(g_skws_mu);
+  for (int i = 0; i < g_skws_n; ++i)
+    if (g_skws[i].dev == dev && g_skws[i].stream == s) {
+      *ws = g_skws[i].ws;
+      *flags = g_skws[i].flags;
+      return true;
+    }
+  if (g_skws_n == 256) return false;
+  cudaStreamCaptureStatus cs;
+  if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) return false;
+  float *w = nullptr;
+  int *f = nullptr;
+  if (cudaMalloc(&w, static_cast<size_t>(num_sms) * 128 * 256 * sizeof(float)) != cudaSuccess) return false;
+  if (cudaMalloc(&f, static_cast<size_t>(num_sms) * sizeof(int)) != cudaSuccess ||
+      cudaMemsetAsync(f, 0, static_cast<size_t>(num_sms) * sizeof(int), s) != cudaSuccess) {
+    cudaFree(w);
+    if (f) cudaFree(f);
+    return false;
+  }
+  g_skws[g_skws_n++] = {dev, s, w, f};
+  *ws = w;
+  *flags = f;
+  return true;
+}
+
 // ----------------------------------------------------------------- TC launch
 template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32>
-hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &td, const TcParams &p,
-                         int dev, const DeviceInfo &di, int max_ctas, cudaStream_t stream) {
+hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &td, const TcParams &p0,
+                         int dev, const DeviceInfo &di, int max_ctas, int sk_mode, bool *sk_used,
+                         cudaStream_t stream) {
   using S = TcShape<BN, CG, OUT_F32>;
   auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32>;
   static int attr_done[kMaxDevices] = {};
@@ -171,10 +236,30 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
     }
     attr_done[dev] = 1;
   }
-  const int tiles = p.num_m_tiles * p.num_n_tiles;
+  const int tiles = p0.num_m_tiles * p0.num_n_tiles;
   int units = max_clusters[dev];
   if (max_ctas > 0) units = std::max(1, std::min(units, max_ctas / CG));
-  const int clusters = std::min(tiles, units);
+  int clusters = std::min(tiles, units);
+  TcParams p = p0;
+  p.dp_tiles = tiles;
+  p.sk_u0 = p.sk_units = 0;
+  p.sk_ws = nullptr;
+  p.sk_flags = nullptr;
+  *sk_used = false;
+  if (S::NH == 1) {
+    const int dp = sk_plan(tiles, units, p.num_k_blocks, sk_mode);
+    float *ws = nullptr;
+    int *flags = nullptr;
+    if (dp >= 0 && units * CG <= di.num_sms && sk_workspace(dev, stream, di.num_sms, &ws, &flags)) {
+      p.dp_tiles = dp;
+      p.sk_u0 = static_cast<int64_t>(dp) * p.num_k_blocks;
+      p.sk_units = static_cast<int64_t>(tiles - dp) * p.num_k_blocks;
+      p.sk_ws = ws;
+      p.sk_flags = flags;
+      clusters = units;
+      *sk_used = true;
+    }
+  }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(clusters * CG);
   cfg.blockDim = dim3(S::THREADS);
@@ -195,10 +280,10 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
 template <int BN, int CG>
 hgemm_status_t dispatch_tc_layout(bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
                                   const CUtensorMap &td, const TcParams &p, int dev, const DeviceInfo &di,
-                                  int max_ctas, cudaStream_t s) {
+                                  int max_ctas, int sk_mode, bool *sk_used, cudaStream_t s) {
 #define HG_CASE(AM, BM_, F)                                                               \
   if (a_mn == AM && b_mn == BM_ && f32 == F)                                              \
-    return launch_tc<BN, CG, AM, BM_, F>(ta, tb, td, p, dev, di, max_ctas, s);
+    return launch_tc<BN, CG, AM, BM_, F>(ta, tb, td, p, dev, di, max_ctas, sk_mode, sk_used, s);
   HG_CASE(false, false, false)
   HG_CASE(false, false, true)
   HG_CASE(false, true, false)
@@ -297,7 +382,8 @@ inline bool is_n(char c) { return c == 'N' || c == 'n'; }
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 // Automatic tile choice: estimated time = waves * per-wave tile cost.
-void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, int forced_cg, int &cg, int &bn) {
+void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, int forced_cg, int sk_mode, int &cg,
+               int &bn) {
   struct Cand { int cg, bn; double eff; };
   // eff: relative per-SM throughput of the tile shape.  Larger tiles move
   // fewer L2->SMEM bytes per FLOP (pair 256x512: 171 FLOP/B, 256x256: 128,
@@ -306,15 +392,17 @@ void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, 
   double best = 1e300;
   for (const Cand &c : cands) {
     if (forced_cg && c.cg != forced_cg) continue;
-    // One 512-column accumulator cannot overlap the epilogue with the next
-    // tile's mainloop; with beta != 0 (C is read in the epilogue) and short K
-    // the exposed epilogue outweighs the bandwidth saving (measured on
-    // BERT-FFN shapes).
-    if (c.bn == 512 && beta_nonzero && K < 4096) continue;
+    // One 512-column accumulator cannot fully overlap the epilogue with the
+    // next tile's mainloop; with beta != 0 (C is read in the epilogue) and
+    // short K that costs a few percent (measured on BERT-FFN shapes).
+    const double eff = (c.bn == 512 && beta_nonzero && K < 4096) ? 0.97 : c.eff;
     const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, c.bn);
     const int64_t units = num_sms / c.cg;
-    const int64_t waves = cdiv(tiles, units);
-    const double t = static_cast<double>(waves) * (128.0 * c.cg * c.bn) / (c.cg * c.eff);
+    double waves = static_cast<double>(cdiv(tiles, units));
+    const int64_t nkb = cdiv(K, 64);
+    if (c.bn <= 256 && sk_plan(tiles, units, nkb, sk_mode) >= 0)  // stream-K: fractional waves
+      waves = static_cast<double>(tiles) / units + sk_overhead_waves(nkb);
+    const double t = waves * (128.0 * c.cg * c.bn) / (c.cg * eff);
     if (t < best * 0.999) { best = t; cg = c.cg; bn = c.bn; }
   }
 }
@@ -340,6 +428,7 @@ hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
     return HGEMM_SUCCESS;
   }
   if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_SPLITK) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->stream_k < 0 || cfg->stream_k > 2) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_SPLITK) {
     if (cfg->block_n != 0 && cfg->block_n != 64 && cfg->block_n != 128) return HGEMM_ERR_INVALID_VALUE;
     if (cfg->splits != 0 && cfg->splits != 2 && cfg->splits != 4 && cfg->splits != 8) return HGEMM_ERR_INVALID_VALUE;
@@ -488,7 +577,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   int cg = 2, bn = 512;
   const int forced_cg = cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
   if (forced_cg && cfg.block_n) { cg = forced_cg; bn = cfg.block_n; }
-  else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, cg, bn);
+  else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, cfg.stream_k, cg, bn);
   const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
 
   CUtensorMap ta, tb;
@@ -504,7 +593,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   if (ok) ok = make_map(&td, C, static_cast<uint64_t>(m), static_cast<uint64_t>(n), ldc, f32 ? 32 : 64, 32, f32);
   if (!ok) return HGEMM_ERR_CUDA;
 
-  TcParams p;
+  TcParams p = {};
   p.M = static_cast<int32_t>(M);
   p.N = static_cast<int32_t>(N);
   p.K = static_cast<int32_t>(k);
@@ -528,17 +617,19 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   p.ldd = ldc;
 
   hgemm_status_t st;
+  bool sk_used = false;
+  const int skm = cfg.stream_k;
   if (cg == 2 && bn == 512)
-    st = dispatch_tc_layout<512, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
+    st = dispatch_tc_layout<512, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
   else if (cg == 2)
-    st = dispatch_tc_layout<256, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
+    st = dispatch_tc_layout<256, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
   else if (bn == 256)
-    st = dispatch_tc_layout<256, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
+    st = dispatch_tc_layout<256, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
   else
-    st = dispatch_tc_layout<128, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, stream);
+    st = dispatch_tc_layout<128, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);
-    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0};
+    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0, sk_used ? 2 : 1};
   }
   return st;
 }

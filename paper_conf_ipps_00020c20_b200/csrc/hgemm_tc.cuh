@@ -53,7 +53,46 @@ struct TcParams {
   void *D;
   int64_t ldd;
   unsigned long long *probe;         // diagnostic (may be null): CTA 0 writes {clk0, ns0, clk1, ns1}
+  // Stream-K: tiles [0, dp_tiles) are processed whole,
+  // round-robin over the clusters; the k-block units [sk_u0, sk_u0 + sk_units)
+  // of the remaining tiles are cut into one contiguous range per cluster.
+  // sk_units == 0: every tile whole (dp_tiles = all tiles).
+  int32_t dp_tiles;
+  int64_t sk_u0, sk_units;
+  float *sk_ws;                      // one 128 x BN FP32 partial-accumulator slot per CTA
+  int *sk_flags;                     // one flag per CTA: 1 = slot published; consumers reset it to 0
 };
+
+// One unit of work of a cluster: k-blocks [kb0, kb1) of cluster tile `tile`.
+struct WorkItem {
+  int tile, kb0, kb1;
+};
+
+__device__ __forceinline__ int64_t sk_begin(const TcParams &p, int c, int G) {
+  return p.sk_u0 + p.sk_units * c / G;
+}
+
+// The i-th work item of cluster c (of G): its whole tiles first, then the
+// tile segments of its stream-K range in k order.  False past the last item.
+__device__ __forceinline__ bool get_item(const TcParams &p, int c, int G, int i, WorkItem &w) {
+  const int n_dp = p.dp_tiles > c ? (p.dp_tiles - c + G - 1) / G : 0;
+  const int nkb = p.num_k_blocks;
+  if (i < n_dp) {
+    w.tile = c + i * G;
+    w.kb0 = 0;
+    w.kb1 = nkb;
+    return true;
+  }
+  if (p.sk_units == 0) return false;
+  const int64_t u0 = sk_begin(p, c, G), u1 = sk_begin(p, c + 1, G);
+  const int t = static_cast<int>(u0 / nkb) + (i - n_dp);
+  const int64_t b = max(u0, static_cast<int64_t>(t) * nkb), e = min(u1, static_cast<int64_t>(t + 1) * nkb);
+  if (b >= e) return false;
+  w.tile = t;
+  w.kb0 = static_cast<int>(b - static_cast<int64_t>(t) * nkb);
+  w.kb1 = static_cast<int>(e - static_cast<int64_t>(t) * nkb);
+  return true;
+}
 
 // UMMA shared-memory descriptor, SWIZZLE_128B, K-major operand.
 // Rows of 128 B (64 FP16 along K); 8-row core groups 1024 B apart (SBO).
@@ -259,9 +298,18 @@ __device__ __forceinline__ void load_c_words(const TcParams &p, uint32_t (&cw)[C
     if (p.probe != nullptr && blockIdx.x == 0 && (it) < 16)                              \
       p.probe[8 + 16 * (it) + (field)] = static_cast<unsigned long long>(clock64());     \
   } while (0)
+// Every CTA: %globaltimer of item `it` < 2 events at p.probe[264 + 8*blockIdx.x + 2 + 3*it + field].
+#define HG_CTRACE(it, field)                                                             \
+  do {                                                                                   \
+    if (p.probe != nullptr && (it) < 2)                                                  \
+      p.probe[264 + 8 * blockIdx.x + 2 + 3 * (it) + (field)] = globaltimer_ns();         \
+  } while (0)
 #else
 #define HG_TRACE(it, field) \
   do {                      \
+  } while (0)
+#define HG_CTRACE(it, field) \
+  do {                       \
   } while (0)
 #endif
 
@@ -297,15 +345,15 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
   uint64_t *empty = full + STAGES;
   uint64_t *tfull = empty + STAGES;      // [ACC][NH]
   uint64_t *tempty = tfull + ACC * NH;   // [ACC][NH]
-  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + ACC * NH);
+  uint64_t *skbar = tempty + ACC * NH;   // [EPI_WARPS][2]: stream-K partial loads
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(skbar + 2 * S::EPI_WARPS);
 
   const uint32_t warp = warp_id();
   const uint32_t lane = lane_id();
   const uint32_t rank = (CG == 2) ? cluster_ctarank() : 0u;
   const int cluster_id = static_cast<int>(blockIdx.x) / CG;
   const int num_clusters = static_cast<int>(gridDim.x) / CG;
-  const int num_tiles = p.num_m_tiles * p.num_n_tiles;
-
+  
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
@@ -323,6 +371,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
           mbar_init(&tempty[a * NH + h], S::EPI_WARPS * CG);
         }
       }
+      for (int b = 0; b < 2 * S::EPI_WARPS; ++b) mbar_init(&skbar[b], 1);
       fence_mbarrier_init();
     }
     __syncwarp();
@@ -333,6 +382,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   unsigned long long probe_clk = 0, probe_ns = 0;
+#ifdef HGEMM_TRACE
+  const unsigned long long cta_t0 = globaltimer_ns();
+#endif
   if (p.probe != nullptr && blockIdx.x == 0 && threadIdx.x == 0) {
     probe_clk = clock64();
     probe_ns = globaltimer_ns();
@@ -346,12 +398,13 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       const uint64_t pol_a = p.l2_hint == 1 ? l2_policy_evict_last() : p.l2_hint == 2 ? l2_policy_evict_normal() : 0;
       const uint64_t pol_b = p.l2_hint == 1 ? l2_policy_evict_first() : p.l2_hint == 2 ? l2_policy_evict_normal() : 0;
       uint32_t stage = 0, phase = 0;
-      for (int t = cluster_id; t < num_tiles; t += num_clusters) {
+      WorkItem wi;
+      for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i) {
         int tm, tn;
-        tile_coords(t, p, tm, tn);
+        tile_coords(wi.tile, p, tm, tn);
         const int a_row = tm * BM * CG + static_cast<int>(rank) * BM;
         const int b_row0 = tn * BN + static_cast<int>(rank) * B_ROWS;
-        for (int kb = 0; kb < p.num_k_blocks; ++kb) {
+        for (int kb = wi.kb0; kb < wi.kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1u);
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
           const uint32_t sb = sa + A_BYTES;
@@ -420,10 +473,11 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
           umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kbl | k) != 0 ? 1u : 0u);
         }
       };
-      const int nkb = p.num_k_blocks;
-      const int end_lag = (NH == 2) ? min(HGEMM_END_LAG, max(nkb - 1, 0)) : 0;
-      const int h1_limit = nkb - end_lag;  // half-1 k-blocks >= h1_limit are issued after the loop
-      for (int t = cluster_id; t < num_tiles; t += num_clusters, ++it) {
+      WorkItem wi;
+      for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i, ++it) {
+        const int nkb = wi.kb1 - wi.kb0;  // k-blocks of this item (kb below counts from its first)
+        const int end_lag = (NH == 2) ? min(HGEMM_END_LAG, max(nkb - 1, 0)) : 0;
+        const int h1_limit = nkb - end_lag;  // half-1 k-blocks >= h1_limit are issued after the loop
         const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
         const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
         const uint32_t d_tmem = tmem_base + buf * BN;
@@ -509,6 +563,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
           umma_commit<CG>(&tfull[buf]);             // accumulator ready for the epilogue
         }
         HG_TRACE(it, 0);
+        HG_CTRACE(it, 0);
 #ifdef HGEMM_TRACE
         if (p.probe != nullptr && blockIdx.x == 0 && it < 16) p.probe[8 + 16 * it + 7] = full_wait;
 #endif
@@ -530,9 +585,42 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     constexpr int VEC = OUT_F32 ? 4 : 8;
     const bool fast = ((p.N & (VEC - 1)) == 0) && (!OUT_F32 || beta == 0.0f);
     constexpr int PKW = OUT_F32 ? EPI_COLS_W : EPI_COLS_W / 2;  // packed result words per thread per half
-    for (int t = cluster_id; t < num_tiles; t += num_clusters, ++it) {
+    // Stream-K partial slots: per CTA slot, per epilogue warp, EPI_COLS_W/32 boxes of
+    // 32 rows x 32 FP32 (4 KB, 16-B chunks swizzled like the staging boxes),
+    // written and read with 1-D bulk copies.
+    constexpr int SK_BOXES = EPI_COLS_W / 32;
+    auto sk_box = [&](int slot_cluster, int j) -> uint8_t * {
+      return reinterpret_cast<uint8_t *>(p.sk_ws) +
+             ((static_cast<int64_t>(slot_cluster * CG + static_cast<int>(rank)) * S::EPI_WARPS + ew) * SK_BOXES + j) *
+                 4096;
+    };
+    // Head items stage the partials in the (then idle) smem ring: 2 x EPI_COLS*128 B per warp.
+    const uint32_t sk_stage = smem_u32(smem) + ew * (2u * EPI_COLS * 128u);
+    static_assert(2u * EPI_COLS * 128u * S::EPI_WARPS <= STAGES * STAGE_BYTES, "stream-K staging");
+    uint32_t sk_uses[2] = {0u, 0u};
+    WorkItem wi;
+    for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i, ++it) {
       int tm, tn;
-      tile_coords(t, p, tm, tn);
+      tile_coords(wi.tile, p, tm, tn);
+      // 0: whole tile; 1: a later k segment of a stream-K tile -> publish FP32
+      // partial; 2: the tile's first segment -> add the later segments' partials
+      const int mode = wi.kb0 > 0 ? 1 : (wi.kb1 < p.num_k_blocks ? 2 : 0);
+      int c_hi = cluster_id + 1;  // mode 2: clusters [cluster_id + 1, c_hi) hold this tile's partials
+      if (mode == 2) {
+        const int64_t tile_end = static_cast<int64_t>(wi.tile + 1) * p.num_k_blocks;
+        while (c_hi < num_clusters && sk_begin(p, c_hi, num_clusters) < tile_end) ++c_hi;
+      }
+      const int n_contrib = c_hi - cluster_id - 1;
+      const int sk_seq = (EPI_COLS_W / EPI_COLS) * n_contrib;  // (chunk, contributor) loads, chunk-major
+      // bulk-load step s of the head's partial stream into staging buffer s & 1
+      auto sk_issue = [&](int s) {
+        const int c = s / n_contrib, q = s - c * n_contrib, b = s & 1;
+        mbar_arrive_expect_tx(&skbar[ew * 2 + b], EPI_COLS * 128);
+#pragma unroll
+        for (int x = 0; x < EPI_COLS / 32; ++x)
+          bulk_load_1d(sk_stage + b * (EPI_COLS * 128) + x * 4096, sk_box(cluster_id + 1 + q, c * (EPI_COLS / 32) + x),
+                       4096, &skbar[ew * 2 + b]);
+      };
       const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
       const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
       const int row_base = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad) * 32;
@@ -541,7 +629,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       // loaded into registers before the accumulator is ready (C does not
       // depend on it), half 1's while half 0 is being stored.
       uint32_t cw[OUT_F32 ? 1 : EPI_COLS_W / 2];
-      const bool pre_c = !OUT_F32 && fast && beta != 0.0f;
+      const bool pre_c = !OUT_F32 && fast && beta != 0.0f && mode == 0;
       if constexpr (!OUT_F32) {
         if (pre_c) {
           load_c_words<EPI_COLS_W>(p, cw, row, tn * BN + cgrp * EPI_COLS_W);
@@ -560,12 +648,29 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       if (warp == 2 && lane == 0) {
         mbar_wait(&tfull[buf * NH], acc_phase);
         HG_TRACE(it, 1);
+        for (int c2 = cluster_id + 1; c2 < c_hi; ++c2) {  // mode 2: wait for the published partials
+          int *f = p.sk_flags + c2 * CG + static_cast<int>(rank);
+          if (ld_acquire_gpu(f) == 0) {
+            const long long t0 = HGEMM_WATCHDOG_CYCLES > 0 ? clock64() : 0;
+            while (ld_acquire_gpu(f) == 0) {
+              __nanosleep(64);
+              watchdog_check(t0);
+            }
+          }
+          *reinterpret_cast<volatile int *>(f) = 0;  // consumed (each flag is set once per launch)
+        }
+        HG_TRACE(it, 12);
+        HG_CTRACE(it, 1);
       }
       named_bar_sync(1, 32 * S::EPI_WARPS);
       tc_fence_after();
       if (warp == 2 && lane == 0) HG_TRACE(it, 8);
+      if (mode == 2 && lane == 0) {  // the partials are published: start streaming them into smem
+        sk_issue(0);
+        if (sk_seq > 1) sk_issue(1);
+      }
       const uint32_t tbase = tmem_base + ((quad * 32u) << 16) + buf * BN;
-      if (fast) {
+      if (fast && mode == 0) {
         // Fast release: read this warp's columns of a whole accumulator half
         // into registers (alpha, beta*C, FP16 packing applied), hand the half
         // back to the MMA warp, then store.
@@ -663,6 +768,53 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
               if (warp == 2) HG_TRACE(it, 2 + h);
             }
           }
+          if (mode == 1) {  // publish this chunk of the partial accumulator: 4-KB boxes, bulk stores
+#pragma unroll
+            for (int x = 0; x < EPI_COLS / 32; ++x) {
+              const uint32_t sbuf = stg + (nstore % EPI_BUFS) * (32u * 128u);
+              if (nstore >= EPI_BUFS) {
+                if (lane == 0) bulk_wait_group_read<EPI_BUFS - 1>();
+                __syncwarp();
+              }
+              const uint32_t rowaddr = sbuf + lane * 128u;
+#pragma unroll
+              for (int q = 0; q < 8; ++q)
+                st_shared_v4(rowaddr + ((q ^ (lane & 7u)) << 4), v[32 * x + 4 * q], v[32 * x + 4 * q + 1],
+                             v[32 * x + 4 * q + 2], v[32 * x + 4 * q + 3]);
+              fence_proxy_async_smem();
+              __syncwarp();
+              if (lane == 0) {
+                bulk_store_1d(sk_box(cluster_id, c * (EPI_COLS / 32) + x), sbuf, 4096);
+                bulk_commit_group();
+              }
+              ++nstore;
+            }
+            continue;
+          }
+          for (int q = 0; q < n_contrib; ++q) {  // mode 2: add the later k segments, in k order
+            const int sidx = c * n_contrib + q, b = sidx & 1;
+            mbar_wait(&skbar[ew * 2 + b], sk_uses[b] & 1u);
+            ++sk_uses[b];
+#pragma unroll
+            for (int x = 0; x < EPI_COLS / 32; ++x) {
+              const uint32_t rowaddr = sk_stage + b * (EPI_COLS * 128) + x * 4096 + lane * 128u;
+#pragma unroll
+              for (int j = 0; j < 8; ++j) {
+                float a0, a1, a2, a3;
+                ld_shared_v4(rowaddr + ((j ^ (lane & 7u)) << 4), a0, a1, a2, a3);
+                const int e = 32 * x + 4 * j;
+                v[e] = __float_as_uint(__uint_as_float(v[e]) + a0);
+                v[e + 1] = __float_as_uint(__uint_as_float(v[e + 1]) + a1);
+                v[e + 2] = __float_as_uint(__uint_as_float(v[e + 2]) + a2);
+                v[e + 3] = __float_as_uint(__uint_as_float(v[e + 3]) + a3);
+              }
+            }
+            __syncwarp();  // every lane has read buffer b
+            if (lane == 0 && sidx + 2 < sk_seq) {
+              fence_proxy_async_smem();
+              sk_issue(sidx + 2);
+            }
+          }
 #ifdef HGEMM_EXP_LDONLY
           if (v[0] == 0x7fc00001u && v[63] == 0x7fc00001u) asm volatile("trap;");  // keep the loads live
           continue;
@@ -725,6 +877,22 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
           emit_row_chunk<OUT_F32, EPI_BUFS>(p, &tmD, stg, nstore, w, col, row, row_base, lane);
         }
       }
+      if (warp == 2 && lane == 0) {
+        HG_TRACE(it, 13);
+        HG_CTRACE(it, 2);
+      }
+      if (mode == 1) {  // every epilogue warp's bulk stores of the slot have completed
+        if (lane == 0) {
+          bulk_wait_group<0>();
+          fence_proxy_async_global();
+        }
+        __syncwarp();
+        named_bar_sync(2, 32 * S::EPI_WARPS);
+        if (warp == 2 && lane == 0) {
+          __threadfence();
+          st_release_gpu(p.sk_flags + cluster_id * CG + static_cast<int>(rank), 1);
+        }
+      }
     }
     if (lane == 0) bulk_wait_group<0>();
   }
@@ -737,6 +905,13 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     p.probe[2] = clock64();
     p.probe[3] = globaltimer_ns();
   }
+#ifdef HGEMM_TRACE
+  // every CTA: {start ns, end ns} at p.probe[264 + 8*blockIdx.x]
+  if (p.probe != nullptr && threadIdx.x == 0) {
+    p.probe[264 + 8 * blockIdx.x] = cta_t0;
+    p.probe[265 + 8 * blockIdx.x] = globaltimer_ns();
+  }
+#endif
   if constexpr (CG == 2) cluster_sync();
   if (warp == 1) {
     tc_fence_after();

@@ -7,7 +7,10 @@ offsets with unchanged leading dimensions:
     C[:, n0:n1]      ->  C + n0*ldc
 No reduction is needed because K is not split, so each rank's slab is
 computed with exactly the single-GPU per-element arithmetic: the
-concatenation of the slabs is bitwise equal to the single-GPU result.
+concatenation of the slabs is bitwise equal to the single-GPU result
+whenever the kernels keep whole tiles (stream-K off, hgemm_config_t
+stream_k = 1; with stream-K a tile split in k sums its FP32 partials in
+k order, which can round differently in the last place).
 
 The one exchange step is the replication of A: an NCCL broadcast from the
 source rank over NVLink/NVSwitch (torch.distributed, backend "nccl" on

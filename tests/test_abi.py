@@ -54,6 +54,8 @@ def test_set_config_validation():
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(9, 0, 0, 0))) == 1
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(2, 96, 0, 0))) == 1
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(2, 128, 8, 0))) == 0
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(2, 128, 0, 0, 0, 3))) == 1   # stream_k 0..2
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 256, 0, 0, 0, 2))) == 0
     assert lib.hgemm_set_config(None) == 0
 
 

@@ -198,14 +198,91 @@ def test_all_kernels_agree_on_random(oracle_mod):
     order inside the tensor core, so tc1/tc2 results are bitwise identical."""
     m, n, k = 700, 900, 640
     base = None
+    from paper_conf_ipps_00020c20_b200 import binding
     for kernel, bn in TC_KERNELS:
-        _use(kernel, bn)
+        binding.set_config(kernel, block_n=bn, stream_k=1)   # whole tiles: no k split anywhere
         case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", out="f32")
         got = case.run_gpu()
         if base is None:
             base = got
         else:
             assert np.array_equal(got.view(np.uint32), base.view(np.uint32)), kernel
+
+
+# (kernel, block_n, max_ctas): cluster counts that give stream-K ranges of
+# 40 / 24 k-blocks (two segments per split tile), 12 (three segments: tiles
+# fewer than clusters) and whole data-parallel waves before the stream-K part.
+SK_CASES = [("tc2", 256, 8), ("tc2", 256, 32), ("tc1", 256, 8), ("tc1", 128, 12), ("tc1", 128, 40),
+            ("tc1", 128, 4)]
+
+
+@pytest.mark.parametrize("kernel,bn,max_ctas", SK_CASES)
+@pytest.mark.parametrize("tA,tB", TRANS)
+@pytest.mark.parametrize("out,beta", [("f16", 0.0), ("f16", 1.0), ("f32", 0.5)])
+def test_stream_k(oracle_mod, kernel, bn, max_ctas, tA, tB, out, beta):
+    """Stream-K: tiles split in k between clusters and summed through the FP32
+    workspace in k order -- within tolerance, deterministic across launches
+    (the flags return to 0 after every launch), padding untouched."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config(kernel, block_n=bn, max_ctas=max_ctas, stream_k=2)
+    m, n, k = 300, 520, 2000
+    C = inputs.uniform_f16(m, n, 7).astype(np.float32 if out == "f32" else np.float16)
+    case = GpuCase(inputs.uniform_f16(m, k, 5), inputs.uniform_f16(k, n, 6), tA, tB, 1.0, beta, C=C, out=out,
+                   pad=(8, 16, 8))
+    a, b, c = case.run_gpu(repeat=3)
+    assert case.stats["last_kernel"] == kernel and case.stats["stream_k"] == 2, case.stats
+    u = np.uint32 if out == "f32" else np.uint16
+    assert np.array_equal(a.view(u), b.view(u)) and np.array_equal(a.view(u), c.view(u))
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, a, r, ab)
+    assert np.all(np.isnan(case.padding(a).astype(np.float32)))
+
+
+@pytest.mark.parametrize("kernel,bn,max_ctas", SK_CASES)
+def test_stream_k_integer_exact(oracle_mod, kernel, bn, max_ctas):
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config(kernel, block_n=bn, max_ctas=max_ctas, stream_k=2)
+    opA = inputs.integer_f16(300, 1984, 3, -4, 4)
+    opB = inputs.integer_f16(1984, 520, 4, -4, 4)
+    case = GpuCase(opA, opB, "T", "N", out="f32")
+    got = case.view(case.run_gpu())
+    assert case.stats["stream_k"] == 2, case.stats
+    _, r, _ = case.oracle(oracle_mod)
+    assert np.array_equal(got.astype(np.float64), r)
+    a, b, expect = inputs.accumulator_width_case(300, 520, 2048)
+    case = GpuCase(a, b, "N", "T", out="f32")
+    assert np.all(case.view(case.run_gpu()) == expect)
+
+
+def test_stream_k_graph_capture(oracle_mod):
+    """Stream-K inside a captured CUDA graph: the workspace is created by an
+    eager call on the stream first; replays reuse it (flags reset each launch)."""
+    import torch
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("tc2", block_n=256, max_ctas=8, stream_k=2)
+    m, n, k = 300, 520, 2000
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", 1.0, 0.0, out="f32")
+    dA = torch.from_numpy(case.A.view(np.int16).copy()).cuda()
+    dB = torch.from_numpy(case.B.view(np.int16).copy()).cuda()
+    dC = torch.full((case.ldc * n,), float("nan"), dtype=torch.float32, device="cuda")
+    s = torch.cuda.Stream()
+    args = (m, n, k, 1.0, dA, case.lda, dB, case.ldb, 0.0, dC, case.ldc, "T", "N", "f32", s.cuda_stream)
+    with torch.cuda.stream(s):
+        binding.hgemm(*args)
+    torch.cuda.synchronize()
+    eager = dC.cpu().numpy().copy()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(s):
+        with torch.cuda.graph(g, stream=s):
+            binding.hgemm(*args)
+    assert binding.get_stats()["stream_k"] == 2
+    for _ in range(3):
+        dC.fill_(float("nan"))
+        g.replay()
+        torch.cuda.synchronize()
+        assert np.array_equal(dC.cpu().numpy().view(np.uint32), eager.view(np.uint32))
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, eager, r, ab)
 
 
 @pytest.mark.parametrize("splits", [2, 4, 8])

@@ -21,7 +21,7 @@ def test_sharded_world1_equals_single_call(beta):
     from paper_conf_ipps_00020c20_b200 import binding, hgemm_sharded, hgemm_sharded_overlapped
     m, n, k = 2048, 1536, 1024
     A, B, C0 = _setup(m, n, k)
-    binding.set_config("tc2", block_n=256)
+    binding.set_config("tc2", block_n=256, stream_k=1)   # whole tiles: the bitwise claim needs one k order
     try:
         ref = C0.clone()
         binding.hgemm(m, n, k, 1.0, A, k, B, k, beta, ref, m, "T", "N", "f16")
