@@ -210,6 +210,70 @@ def cpu_baseline(workload, budget_s=12.0):
             "sample": f"{ms} x {ns} block of C with the full k = {k} of {workload} ({dt:.1f} s)"}
 
 
+# ------------------------------------------------------------------ roofline
+def alg_bytes(m, n, k, beta, esz):
+    """Minimum HBM traffic of one launch: read A and B once, write C (and read it if beta != 0)."""
+    return 2.0 * (m * k + k * n) + esz * m * n * (2 if beta != 0 else 1)
+
+
+def roofline_entry(m, n, k, beta, esz, ms, peaks, traffic):
+    """Roofline of the launch: tensor-bound when its intensity 2mnk / alg_bytes is above the
+    ridge (measured bf16 TFLOP/s / measured HBM GB/s), HBM-bound below it."""
+    flops = 2.0 * m * n * k
+    byts = alg_bytes(m, n, k, beta, esz)
+    ridge = peaks["tflops_burst"] * 1e12 / (peaks["hbm_gbs"] * 1e9)
+    tb = traffic.get("bytes_per_launch") if isinstance(traffic, dict) else None
+    if flops / byts >= ridge:
+        a = flops / (ms * 1e-3) / 1e12
+        return {"bound": "tensor", "achieved": a, "peak": peaks["tflops_burst"], "unit": UNIT,
+                "frac": a / peaks["tflops_burst"], "traffic": tb, "traffic_detail": traffic,
+                "peak_source": peaks["source"] + " burst (kernel timed alone)",
+                "algorithmic": f"2*m*n*k = {flops:.4e} FLOP per launch (intensity {flops / byts:.0f} FLOP/B, "
+                               f"ridge {ridge:.0f})"}
+    a = byts / (ms * 1e-3) / 1e9
+    return {"bound": "hbm", "achieved": a, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+            "frac": a / peaks["hbm_gbs"], "traffic": tb, "traffic_detail": traffic,
+            "peak_source": peaks["source"],
+            "algorithmic": f"2(mk+kn) + s_out*mn*(1+[beta!=0]) = {byts:.4e} B per launch "
+                           f"(intensity {flops / byts:.0f} FLOP/B, ridge {ridge:.0f})"}
+
+
+def skinny_roofline(dev, flush, peaks, reps=20):
+    """BJ configs[3]: M=16384, N in {64,128,256}, K=4096 (TN, FP16 out), device-resident,
+    L2 flushed between launches; achieved GB/s of the algorithmic bytes vs the HBM peak."""
+    import torch
+    from paper_conf_ipps_00020c20_b200 import binding, inputs
+    out = {}
+    for name in ("cfg4_skinny_n64", "cfg4_skinny_n128", "cfg4_skinny_n256"):
+        m, n, k, tA, tB, alpha, beta, o = inputs.WORKLOADS[name]
+        g = torch.Generator(device=dev).manual_seed(99)
+        sa, sb = inputs.stored_shape(m, k, tA), inputs.stored_shape(k, n, tB)
+        A = (torch.rand(sa[1], sa[0], generator=g, device=dev) * 2 - 1).half()
+        B = (torch.rand(sb[1], sb[0], generator=g, device=dev) * 2 - 1).half()
+        C = torch.empty(n, m, dtype=torch.float16, device=dev)
+
+        def call():
+            binding.hgemm(m, n, k, alpha, A, sa[0], B, sb[0], beta, C, m, tA, tB, o)
+        for _ in range(3):
+            call()
+        ts = []
+        for _ in range(reps):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            call()
+            e1.record()
+            ts.append((e0, e1))
+        torch.cuda.synchronize()
+        ms = statistics.mean(a.elapsed_time(b) for a, b in ts)
+        r = roofline_entry(m, n, k, beta, 2, ms, peaks, None)
+        st = binding.get_stats()
+        out[name] = {"ms": ms, "bound": r["bound"], "achieved": r["achieved"], "unit": r["unit"],
+                     "frac": r["frac"], "TFLOP/s": 2.0 * m * n * k / (ms * 1e-3) / 1e12,
+                     "kernel": f"{st['last_kernel']}/{st['block_n']}" + (f" split {st['splits']}" if st['splits'] else "")}
+    return out
+
+
 # ------------------------------------------------------------------ our arm
 def run_ours(args, world, rank, local):
     import torch
@@ -229,11 +293,12 @@ def run_ours(args, world, rank, local):
             dist.init_process_group(backend)
     lib = binding.load_library()
     m, n_cfg, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[args.workload]
+    if args.beta is not None:       # experiments only: override the workload's beta
+        beta = args.beta
     strong = args.workload in inputs.STRONG_SCALING
-    if args.kernel != "auto":
-        binding.set_config(args.kernel, block_n=args.block_n, group_m=args.group_m)
-    elif args.group_m:
-        binding.set_config("auto", group_m=args.group_m)
+    if args.kernel != "auto" or args.group_m or args.stream_k or args.splits:
+        binding.set_config(args.kernel, block_n=args.block_n, group_m=args.group_m, stream_k=args.stream_k,
+                           splits=args.splits)
     # weak scaling: every rank owns an n_cfg-wide slab (global n = n_cfg * world);
     # strong scaling (config 5): the global n_cfg columns are split over the ranks.
     n_glob = n_cfg if strong else n_cfg * world
@@ -417,6 +482,11 @@ def run_ours(args, world, rank, local):
         except Exception as e:  # pragma: no cover
             cublas = {"error": f"{type(e).__name__}: {e}"}
 
+    # the HBM-bound skinny configs (BJ configs[3]) against the HBM roofline (north_star (5))
+    side = None
+    if rank == 0 and world == 1 and not args.no_side and args.workload == "cfg2_8192_TN_f16":
+        side = skinny_roofline(dev, flush, peaks)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_baseline(args.workload, budget_s=args.cpu_budget)
@@ -424,6 +494,7 @@ def run_ours(args, world, rank, local):
     if rank == 0:
         peak = peaks["tflops_burst"]
         traffic = load_traffic(args.workload)
+        roof = roofline_entry(m, n_rank, k, beta, esz, ms_local, peaks, traffic)
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
@@ -434,16 +505,14 @@ def run_ours(args, world, rank, local):
                        "kernel": stats, "l2": "flushed between steps (256 MiB write, outside the events)",
                        "parallelism": f"n-slab x{world}" if world > 1 else "single GPU"},
             "pct_of_peak": 100.0 * value / world / peak,
-            "roofline": {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": UNIT,
-                         "frac": achieved / peak, "traffic": traffic,
-                         "peak_source": peaks["source"] + " burst (kernel timed alone)",
-                         "algorithmic": f"2*m*n*k = {flops_rank:.4e} FLOP per launch"},
+            "roofline": roof,
             "gpu_launches": int(launches),
             "clocks": clk,
             "e2e": e2e,
             "cublas": cublas,
             "cpu_baseline": cpu,
             "collective": coll,
+            "hbm_bound_configs": side,
             "step_ms": {"min": min(step_ms), "median": statistics.median(step_ms), "max": max(step_ms)},
         }
         print(json.dumps(line), flush=True)
@@ -461,7 +530,10 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="cfg2_8192_TN_f16")
-    ap.add_argument("--kernel", default="auto", choices=["auto", "tc1", "tc2", "simt"])
+    ap.add_argument("--kernel", default="auto", choices=["auto", "tc1", "tc2", "simt", "splitk"])
+    ap.add_argument("--stream-k", type=int, default=0, help="0 auto, 1 never, 2 always (experiments)")
+    ap.add_argument("--splits", type=int, default=0, help="split-K cluster size (experiments)")
+    ap.add_argument("--beta", type=float, default=None, help="override the workload's beta (experiments)")
     ap.add_argument("--block-n", type=int, default=0)
     ap.add_argument("--group-m", type=int, default=0)
     ap.add_argument("--ref-budget", type=float, default=60.0, help="seconds of oracle work for --impl reference")
@@ -470,6 +542,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cublas", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-side", action="store_true", help="skip the skinny-shape HBM roofline report")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     world, rank, local = dist_env()

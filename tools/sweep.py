@@ -10,7 +10,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 def run(args, env=None, label=""):
     e = dict(os.environ)
     e.update(env or {})
-    p = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--no-cpu", "--no-e2e", *args],
+    p = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--no-cpu", "--no-e2e", "--no-side", *args],
                        capture_output=True, text=True, env=e, timeout=600)
     lines = [l for l in p.stdout.splitlines() if l.startswith("{")]
     if not lines:
