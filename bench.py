@@ -11,7 +11,7 @@ into TMEM, alpha/beta epilogue) over one batch of synthetic input.
           8192-column slab of C (global n = 8192*N) and A is replicated by
           an NCCL broadcast (timed and reported separately, "collective").
 Timing: W untimed warm-up steps, then K steps, each bracketed by CUDA events
-on the launching stream; L2 is flushed (a 256 MiB write) between steps,
+on the launching stream; L2 is flushed (a 256 MiB write + a 256 MiB read) between steps,
 outside the events; a barrier + synchronize bracket the timed region; the
 time is the max over ranks.  Rank 0 prints ONE JSON line.
 
@@ -210,6 +210,25 @@ def cpu_baseline(workload, budget_s=12.0):
             "sample": f"{ms} x {ns} block of C with the full k = {k} of {workload} ({dt:.1f} s)"}
 
 
+# ------------------------------------------------------------------ L2 flush
+class L2Flush:
+    """Cold-L2 state between timed launches, outside the events: write a 256 MiB buffer
+    (2x the 126 MB L2), then read a second 256 MiB buffer so that the dirty lines of the
+    write are written back here rather than inside the next timed launch (the L2 is
+    left holding clean, unrelated lines)."""
+
+    def __init__(self, dev):
+        import torch
+        self.w = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+        self.r = torch.zeros(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+        self.sink = torch.empty((), dtype=torch.float32, device=dev)
+
+    def __call__(self):
+        import torch
+        self.w.zero_()
+        torch.sum(self.r, dim=0, out=self.sink)
+
+
 # ------------------------------------------------------------------ roofline
 def alg_bytes(m, n, k, beta, esz):
     """Minimum HBM traffic of one launch: read A and B once, write C (and read it if beta != 0)."""
@@ -258,7 +277,7 @@ def skinny_roofline(dev, flush, peaks, reps=20):
             call()
         ts = []
         for _ in range(reps):
-            flush.zero_()
+            flush()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
             call()
@@ -318,7 +337,7 @@ def run_ours(args, world, rank, local):
     if beta != 0:
         C.uniform_(-1, 1)
     lda, ldb = sa[0], sb_rank[0]
-    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    flush = L2Flush(dev)
     stream = torch.cuda.current_stream()
 
     # the sharded path's one collective: replicate A (rank 0's copy) over NCCL, timed separately
@@ -366,7 +385,7 @@ def run_ours(args, world, rank, local):
                       broadcast=False, local_slabs=True, stream=stream.cuda_stream)
 
     for _ in range(args.warmup):
-        flush.zero_()
+        flush()
         step()
     torch.cuda.synchronize()
     if world > 1:
@@ -378,7 +397,7 @@ def run_ours(args, world, rank, local):
     evs = []
     probe = torch.zeros(4 * args.steps, dtype=torch.int64, device=dev)   # in-kernel SM clock probe
     for i in range(args.steps):
-        flush.zero_()                                   # L2 flush, outside the events
+        flush()                                   # L2 flush, outside the events
         binding.set_probe(probe[4 * i:])
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
@@ -466,7 +485,7 @@ def run_ours(args, world, rank, local):
             torch.cuda.synchronize()
             ts = []
             for _ in range(max(3, min(args.steps, 20))):
-                flush.zero_()
+                flush()
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record()
                 cub()
@@ -502,7 +521,7 @@ def run_ours(args, world, rank, local):
             "vs_baseline": None, "dtype": "f16xf16->f32 (" + out + " out)", "data": "synthetic",
             "config": {"workload": args.workload, "m": m, "n": n_glob, "k": k, "n_per_gpu_rank0": n_rank,
                        "layout": tA + tB, "alpha": alpha, "beta": beta, "out": out,
-                       "kernel": stats, "l2": "flushed between steps (256 MiB write, outside the events)",
+                       "kernel": stats, "l2": "flushed between steps, outside the events: 256 MiB write, then a 256 MiB read so the write's dirty lines are written back before the timed launch",
                        "parallelism": f"n-slab x{world}" if world > 1 else "single GPU"},
             "pct_of_peak": 100.0 * value / world / peak,
             "roofline": roof,
@@ -530,7 +549,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="cfg2_8192_TN_f16")
-    ap.add_argument("--kernel", default="auto", choices=["auto", "tc1", "tc2", "simt", "splitk"])
+    ap.add_argument("--kernel", default="auto", choices=["auto", "tc1", "tc2", "simt", "splitk", "stream"])
     ap.add_argument("--stream-k", type=int, default=0, help="0 auto, 1 never, 2 always (experiments)")
     ap.add_argument("--splits", type=int, default=0, help="split-K cluster size (experiments)")
     ap.add_argument("--beta", type=float, default=None, help="override the workload's beta (experiments)")

@@ -102,14 +102,19 @@ typedef enum {
     HGEMM_KERNEL_SIMT = 1,       /* CUDA-core fallback (always available) */
     HGEMM_KERNEL_TC_1SM = 2,     /* tcgen05 cta_group::1, tile 128 x block_n */
     HGEMM_KERNEL_TC_2SM = 3,     /* tcgen05 cta_group::2 (CTA pair), tile 256 x block_n (256 or 512) */
-    HGEMM_KERNEL_SPLITK = 4      /* tcgen05 cta_group::1, tile 128 x block_n (64 or 128), K split over a
+    HGEMM_KERNEL_SPLITK = 4,     /* tcgen05 cta_group::1, tile 128 x block_n (64 or 128), K split over a
                                     cluster of `splits` CTAs, reduced through distributed shared memory */
+    HGEMM_KERNEL_STREAM = 5      /* HBM-streaming tcgen05 kernel for skinny shapes: n <= 256, transA 'T',
+                                    transB 'N' (both operands K-contiguous); one persistent CTA per SM,
+                                    each owning column chunks of C^T of block_n (multiple of 16) rows of op(A);
+                                    other shapes/layouts fall back to the automatic choice */
 } hgemm_kernel_t;
 
 typedef struct {
     int32_t kernel;    /* hgemm_kernel_t */
     int32_t block_n;   /* tile width along the output's contiguous dim: 128, 256 (1-SM, 2-SM) or
-                          512 (2-SM only); 0 = auto */
+                          512 (2-SM only); HGEMM_KERNEL_STREAM: chunk width, a multiple of 16 in
+                          [16, 256] (n <= 128) or [16, 128] (n <= 256); 0 = auto */
     int32_t group_m;   /* L2 raster group height in tiles (0 = auto) */
     int32_t max_ctas;  /* cap on persistent CTAs (0 = all SMs) */
     int32_t splits;    /* HGEMM_KERNEL_SPLITK: K splits per tile, 2, 4 or 8 (0 = auto) */

@@ -17,7 +17,7 @@ HEADER = os.path.join(_ROOT, "include", "hgemm.h")
 
 HGEMM_OUT_F16 = 0
 HGEMM_OUT_F32 = 1
-HGEMM_KERNEL = {"auto": 0, "simt": 1, "tc1": 2, "tc2": 3, "splitk": 4}
+HGEMM_KERNEL = {"auto": 0, "simt": 1, "tc1": 2, "tc2": 3, "splitk": 4, "stream": 5}
 
 _lib = None
 

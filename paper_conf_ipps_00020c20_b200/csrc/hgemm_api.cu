@@ -20,6 +20,7 @@
 #include "../../include/hgemm.h"
 #include "hgemm_simt.cuh"
 #include "hgemm_splitk.cuh"
+#include "hgemm_stream.cuh"
 #include "hgemm_tc.cuh"
 
 namespace {
@@ -377,6 +378,45 @@ bool choose_splitk(int64_t M, int64_t N, int64_t K, int num_sms, int &bn, int &s
   }
   return spl != 0;
 }
+// ----------------------------------------------------------------- HBM-streaming launch
+template <int MT, bool F32>
+hgemm_status_t launch_stream(const CUtensorMap &ta, const CUtensorMap &tb, const hg::StreamParams &p, int grid,
+                             int dev, cudaStream_t stream) {
+  auto kern = hg::hgemm_stream_kernel<MT, F32>;
+  static int attr_done[kMaxDevices] = {};
+  if (!attr_done[dev]) {
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, hg::kStreamSmemBytes) !=
+        cudaSuccess)
+      return HGEMM_ERR_CUDA;
+    attr_done[dev] = 1;
+  }
+  const uint32_t smem = p.stages * p.stage_bytes + 1024u /*align*/ + 512u /*barriers*/;
+  kern<<<static_cast<unsigned>(grid), 192, smem, stream>>>(ta, tb, p);
+  if (cudaPeekAtLastError() != cudaSuccess) return HGEMM_ERR_CUDA;
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+  return HGEMM_SUCCESS;
+}
+
+// Chunk width for the streaming kernel: the smallest number of chunk waves over
+// the SMs, then the widest chunk (fewest Ak re-reads) among those.
+int stream_chunk(int64_t N, int mt, int num_sms) {
+  const int cw_max = mt == 1 ? 256 : 128;
+  int best = cw_max;
+  int64_t best_w = INT64_MAX;
+  for (int cw = cw_max; cw >= 16; cw -= 16) {
+    const int64_t chunks = (N + cw - 1) / cw;
+    const int64_t waves = (chunks + num_sms - 1) / num_sms;
+    if (waves * cw < best_w) { best_w = waves * cw; best = cw; }
+  }
+  return best;
+}
+
+// The streaming kernel takes HBM-bound skinny shapes: M (= n) <= 256 with an
+// N (= m) that gives every SM at least 4 chunk rows of 16.
+inline bool choose_stream(int64_t M, int64_t N, int64_t K, int num_sms) {
+  return M <= 256 && N >= static_cast<int64_t>(num_sms) * 64 && K >= 256;
+}
+
 inline bool is_t(char c) { return c == 'T' || c == 't'; }
 inline bool is_n(char c) { return c == 'N' || c == 'n'; }
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
@@ -393,9 +433,10 @@ void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, 
   for (const Cand &c : cands) {
     if (forced_cg && c.cg != forced_cg) continue;
     // One 512-column accumulator cannot fully overlap the epilogue with the
-    // next tile's mainloop; with beta != 0 (C is read in the epilogue) and
-    // short K that costs a few percent (measured on BERT-FFN shapes).
-    const double eff = (c.bn == 512 && beta_nonzero && K < 4096) ? 0.97 : c.eff;
+    // next tile's mainloop, and its staging (one box per epilogue warp) cannot
+    // prefetch a whole accumulator half of C; with beta != 0 that costs ~3% at
+    // K = 8192 and ~7% at K = 1024 (BERT-FFN shapes).
+    const double eff = (c.bn == 512 && beta_nonzero) ? (K < 4096 ? 0.90 : 0.97) : c.eff;
     const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, c.bn);
     const int64_t units = num_sms / c.cg;
     double waves = static_cast<double>(cdiv(tiles, units));
@@ -427,7 +468,7 @@ hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
     g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
     return HGEMM_SUCCESS;
   }
-  if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_SPLITK) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_STREAM) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->stream_k < 0 || cfg->stream_k > 2) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_SPLITK) {
     if (cfg->block_n != 0 && cfg->block_n != 64 && cfg->block_n != 128) return HGEMM_ERR_INVALID_VALUE;
@@ -437,6 +478,12 @@ hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
     return HGEMM_SUCCESS;
   }
   if (cfg->splits != 0) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->kernel == HGEMM_KERNEL_STREAM) {
+    if (cfg->block_n < 0 || cfg->block_n > 256 || cfg->block_n % 16 != 0) return HGEMM_ERR_INVALID_VALUE;
+    if (cfg->group_m < 0 || cfg->max_ctas < 0) return HGEMM_ERR_INVALID_VALUE;
+    g_cfg = *cfg;
+    return HGEMM_SUCCESS;
+  }
   if (cfg->block_n != 0 && cfg->block_n != 128 && cfg->block_n != 256 && cfg->block_n != 512)
     return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_TC_2SM && cfg->block_n == 128) return HGEMM_ERR_INVALID_VALUE;
@@ -530,6 +577,47 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   const int64_t M = n, N = m;  // kernel coordinates (D = C^T)
   const bool a_mn = tB;   // Ak = op(B)^T: 'T' -> rows of Ak contiguous along M
   const bool b_mn = !tA;  // Bk = op(A):   'N' -> rows of Bk contiguous along N
+
+  // ---------------------------------------------------------- HBM streaming (skinny, TN)
+  if (!a_mn && !b_mn && M <= 256 &&
+      ((cfg.kernel == HGEMM_KERNEL_STREAM) ||
+       (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream(M, N, k, di.num_sms)))) {
+    const int mt = M <= 128 ? 1 : 2;
+    int cw = cfg.kernel == HGEMM_KERNEL_STREAM && cfg.block_n ? cfg.block_n : stream_chunk(N, mt, di.num_sms);
+    if (mt == 2 && cw > 128) cw = 128;
+    CUtensorMap ta, tb;
+    bool ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
+    if (ok) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, cw);
+    if (!ok) return HGEMM_ERR_CUDA;
+    hg::StreamParams p = {};
+    p.M = static_cast<int32_t>(M);
+    p.N = static_cast<int32_t>(N);
+    p.K = static_cast<int32_t>(k);
+    p.cw = cw;
+    p.num_chunks = static_cast<int32_t>(cdiv(N, cw));
+    p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
+    p.stage_bytes = static_cast<uint32_t>(mt) * 16384u + static_cast<uint32_t>(cw) * 128u;
+    p.stages = static_cast<int32_t>(std::min<uint32_t>(hg::kStreamMaxStages,
+                                                       (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
+    p.k_rot = 1;
+    if (const char *e = std::getenv("HGEMM_STREAM_ROT")) p.k_rot = std::atoi(e);  // experiments
+    p.alpha = alpha;
+    p.beta = beta;
+    p.D = C;
+    p.ldd = ldc;
+    int grid = static_cast<int>(std::min<int64_t>(p.num_chunks, di.num_sms));
+    if (cfg.max_ctas > 0) grid = std::min(grid, cfg.max_ctas);
+    hgemm_status_t st;
+    if (mt == 1) st = f32 ? launch_stream<1, true>(ta, tb, p, grid, dev, stream)
+                          : launch_stream<1, false>(ta, tb, p, grid, dev, stream);
+    else st = f32 ? launch_stream<2, true>(ta, tb, p, grid, dev, stream)
+                  : launch_stream<2, false>(ta, tb, p, grid, dev, stream);
+    if (st == HGEMM_SUCCESS) {
+      std::lock_guard<std::mutex> lk(g_mu);
+      g_last = {HGEMM_KERNEL_STREAM, cw, 0, grid, 0, 0};
+    }
+    return st;
+  }
 
   // ---------------------------------------------------------- split-K (under-filled shapes)
   {

@@ -247,44 +247,6 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
   ++nstore;
 }
 
-// Load COLS FP16 values of C (this thread's row, columns [col, col+COLS)) as
-// COLS/2 packed words; 16-B granules outside [0, N) or rows >= M read as 0.
-// Requires N % 8 == 0 (the fast epilogue path's precondition).
-template <int COLS>
-__device__ __forceinline__ void load_c_words(const TcParams &p, uint32_t (&cw)[COLS / 2], int row, int col) {
-  const __half *src = static_cast<const __half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
-#ifdef HGEMM_C_EVICT_FIRST
-  // 32-B loads (N % 8 == 0 and 16-B aligned rows; a 32-B load needs 32-B
-  // alignment, which holds when ldd % 16 == 0 -- otherwise 16-B granules)
-  if ((p.ldd & 15) == 0 && (reinterpret_cast<uintptr_t>(p.D) & 31) == 0) {
-#pragma unroll
-    for (int q = 0; q < COLS / 16; ++q) {
-      uint32_t v[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
-      if (row < p.M && col + 16 * q < p.N) {
-        if (col + 16 * q + 16 <= p.N) {
-          ld_global_v8_evict_first(src + 16 * q, v);
-        } else {
-          const uint4 h = reinterpret_cast<const uint4 *>(src + 16 * q)[0];
-          v[0] = h.x; v[1] = h.y; v[2] = h.z; v[3] = h.w;
-        }
-      }
-#pragma unroll
-      for (int e = 0; e < 8; ++e) cw[8 * q + e] = v[e];
-    }
-    return;
-  }
-#endif
-#pragma unroll
-  for (int q = 0; q < COLS / 8; ++q) {
-    uint4 v = make_uint4(0u, 0u, 0u, 0u);
-    if (row < p.M && col + 8 * q < p.N) v = reinterpret_cast<const uint4 *>(src)[q];
-    cw[4 * q + 0] = v.x;
-    cw[4 * q + 1] = v.y;
-    cw[4 * q + 2] = v.z;
-    cw[4 * q + 3] = v.w;
-  }
-}
-
 // k-blocks by which accumulator half 1 trails half 0 at the end of a 512-wide tile
 #ifndef HGEMM_END_LAG
 #define HGEMM_END_LAG 2
@@ -579,11 +541,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     const float alpha = p.alpha, beta = p.beta;
     uint32_t nstore = 0;
     int it = 0;
-    // Fast release applies to every case except FP32 output with beta != 0
-    // (whose C half would not fit in registers) and an N that is not a
-    // multiple of 16 B (TMA store granularity).
+    // Fast release (beta == 0) and c_tma (beta != 0) need an N that is a
+    // multiple of 16 B (TMA store granularity); other cases go chunk by chunk.
     constexpr int VEC = OUT_F32 ? 4 : 8;
-    const bool fast = ((p.N & (VEC - 1)) == 0) && (!OUT_F32 || beta == 0.0f);
+    const bool fast = ((p.N & (VEC - 1)) == 0) && beta == 0.0f;
     constexpr int PKW = OUT_F32 ? EPI_COLS_W : EPI_COLS_W / 2;  // packed result words per thread per half
     // Stream-K partial slots: per CTA slot, per epilogue warp, EPI_COLS_W/32 boxes of
     // 32 rows x 32 FP32 (4 KB, 16-B chunks swizzled like the staging boxes),
@@ -625,22 +586,26 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
       const int row_base = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad) * 32;
       const int row = row_base + static_cast<int>(lane);
-      // FP16 output with beta != 0: this warp's C for accumulator half 0 is
-      // loaded into registers before the accumulator is ready (C does not
-      // depend on it), half 1's while half 0 is being stored.
-      uint32_t cw[OUT_F32 ? 1 : EPI_COLS_W / 2];
-      const bool pre_c = !OUT_F32 && fast && beta != 0.0f && mode == 0;
-      if constexpr (!OUT_F32) {
-        if (pre_c) {
-          load_c_words<EPI_COLS_W>(p, cw, row, tn * BN + cgrp * EPI_COLS_W);
-          // half 1's C is loaded only after half 0 is stored: pull it into L2 now
-          if (NH > 1 && row < p.M) {
-            const __half *c1 = static_cast<const __half *>(p.D) + static_cast<int64_t>(row) * p.ldd + tn * BN +
-                               UMMA_N + cgrp * EPI_COLS_W;
+      // beta != 0 (whole tiles, N a multiple of 16 B): C is brought into this warp's
+      // staging boxes by TMA before the accumulator is ready, combined in place and
+      // stored from the same box ("c_tma").  The first EPI_BUFS boxes are loaded now,
+      // the rest are prefetched into L2 and loaded when their box is free.
+      constexpr int NB = EPI_COLS_W / EPI_COLS;  // staging boxes per warp per accumulator half
+      constexpr int NBT = NH * NB;               // ... per tile
+      const bool c_tma = beta != 0.0f && mode == 0 && (p.N & (VEC - 1)) == 0;
+      const uint32_t s0 = nstore;
+      auto box_col = [&](int j) { return tn * BN + (j / NB) * UMMA_N + cgrp * EPI_COLS_W + (j % NB) * EPI_COLS; };
+      auto c_load = [&](int j) {
+        const uint32_t b = (s0 + static_cast<uint32_t>(j)) % EPI_BUFS;
+        mbar_arrive_expect_tx(&skbar[ew * 2 + b], 32u * 128u);
+        tma_load_2d(&tmD, stg + b * (32u * 128u), smem_u32(&skbar[ew * 2 + b]), box_col(j), row_base, 0);
+      };
+      if (c_tma && lane == 0) {
+        bulk_wait_group_read<0>();  // earlier stores have read every staging box of this warp
 #pragma unroll
-            for (int q = 0; q < EPI_COLS_W * 2 / 128; ++q)
-              if (tn * BN + UMMA_N + cgrp * EPI_COLS_W + q * 64 < p.N) prefetch_l2(c1 + q * 64);
-          }
+        for (int j = 0; j < NBT; ++j) {
+          if (j < EPI_BUFS) c_load(j);
+          else tma_prefetch_l2_2d(&tmD, box_col(j), row_base);
         }
       }
       // One thread polls the accumulator barrier; the other epilogue warps
@@ -670,10 +635,79 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         if (sk_seq > 1) sk_issue(1);
       }
       const uint32_t tbase = tmem_base + ((quad * 32u) << 16) + buf * BN;
+      if (c_tma) {
+        // per staging box: TMEM -> registers, wait for its C box, alpha*acc + beta*C
+        // in FP32 in place, TMA store; a half goes back to the MMA warp after its
+        // last box's TMEM read, a box after its store has read it takes the next C box
+#pragma unroll 1
+        for (int h = 0; h < NH; ++h) {
+          if (h > 0) {
+            if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
+            __syncwarp();
+            tc_fence_after();
+          }
+#pragma unroll 1
+          for (int c = 0; c < NB; ++c) {
+            const int j = h * NB + c;
+            const int colt = h * UMMA_N + cgrp * EPI_COLS_W + c * EPI_COLS;
+            uint32_t v[EPI_COLS];
+            tmem_ld_32x32b_x32(tbase + colt, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+            if constexpr (EPI_COLS == 64) tmem_ld_32x32b_x32(tbase + colt + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+            tmem_ld_wait();
+            if (c == NB - 1) {
+              tc_fence_before();
+              __syncwarp();
+              if (lane == 0) {
+                if constexpr (CG == 2) mbar_arrive_cluster_relaxed(tempty_addr + (buf * NH + h) * 8);
+                else mbar_arrive_relaxed(&tempty[buf * NH + h]);
+                if (warp == 2) HG_TRACE(it, 2 + h);
+              }
+            }
+            const uint32_t b = (s0 + static_cast<uint32_t>(j)) % EPI_BUFS;
+            mbar_wait(&skbar[ew * 2 + b], sk_uses[b] & 1u);
+            ++sk_uses[b];
+            const uint32_t sbuf = stg + b * (32u * 128u);
+            const uint32_t rowaddr = sbuf + lane * 128u;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+              const uint32_t addr = rowaddr + ((q ^ (lane & 7u)) << 4);
+              uint32_t cv[4];
+              ld_shared_v4_u32(addr, cv);
+              uint32_t w[4];
+              if constexpr (OUT_F32) {
+#pragma unroll
+                for (int e = 0; e < 4; ++e)
+                  w[e] = __float_as_uint(fmaf(beta, __uint_as_float(cv[e]), alpha * __uint_as_float(v[4 * q + e])));
+              } else {
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                  const float2 cf = __half22float2(*reinterpret_cast<const __half2 *>(&cv[e]));
+                  const int jj = 4 * q + e;
+                  w[e] = pack_half2(fmaf(beta, cf.x, alpha * __uint_as_float(v[2 * jj])),
+                                    fmaf(beta, cf.y, alpha * __uint_as_float(v[2 * jj + 1])));
+                }
+              }
+              st_shared_v4(addr, w[0], w[1], w[2], w[3]);
+            }
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) {
+              tma_store_2d(&tmD, sbuf, tn * BN + colt, row_base);
+              bulk_commit_group();
+              if (j + EPI_BUFS < NBT) {
+                bulk_wait_group_read<0>();  // this box's store has read it: load the next C box
+                c_load(j + EPI_BUFS);
+              }
+            }
+          }
+        }
+        nstore = s0 + NBT;
+        continue;
+      }
       if (fast && mode == 0) {
-        // Fast release: read this warp's columns of a whole accumulator half
-        // into registers (alpha, beta*C, FP16 packing applied), hand the half
-        // back to the MMA warp, then store.
+        // Fast release (beta == 0): read this warp's columns of a whole accumulator
+        // half into registers (alpha and FP16 packing applied), hand the half back
+        // to the MMA warp, then store.
 #pragma unroll 1
         for (int h = 0; h < NH; ++h) {
           if (h > 0) {  // each half has its own tmem_full barrier
@@ -683,44 +717,21 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
           }
           uint32_t pk[PKW];
           const int c0 = h * UMMA_N + cgrp * EPI_COLS_W;  // first tile column of this warp
-          if (!pre_c) {
-            // two TMEM loads in flight per wait (no C registers live in this case)
+          // two TMEM loads in flight per wait
 #pragma unroll
-            for (int b = 0; b < EPI_COLS_W / 64; ++b) {
-              uint32_t v[64];
-              tmem_ld_32x32b_x32(tbase + c0 + b * 64, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
-              tmem_ld_32x32b_x32(tbase + c0 + b * 64 + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
-              tmem_ld_wait();
-              if (warp == 2 && lane == 0 && h == 0 && b == 0) HG_TRACE(it, 9);
-              if constexpr (OUT_F32) {
-#pragma unroll
-                for (int j = 0; j < 64; ++j) pk[b * 64 + j] = __float_as_uint(alpha * __uint_as_float(v[j]));
-              } else {
-#pragma unroll
-                for (int j = 0; j < 32; ++j)
-                  pk[b * 32 + j] = pack_half2(alpha * __uint_as_float(v[2 * j]), alpha * __uint_as_float(v[2 * j + 1]));
-              }
-            }
-          } else
-#pragma unroll
-          for (int b = 0; b < EPI_COLS_W / 32; ++b) {
-            uint32_t v[32];
-            tmem_ld_32x32b_x32(tbase + c0 + b * 32, v);
+          for (int b = 0; b < EPI_COLS_W / 64; ++b) {
+            uint32_t v[64];
+            tmem_ld_32x32b_x32(tbase + c0 + b * 64, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+            tmem_ld_32x32b_x32(tbase + c0 + b * 64 + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
             tmem_ld_wait();
+            if (warp == 2 && lane == 0 && h == 0 && b == 0) HG_TRACE(it, 9);
             if constexpr (OUT_F32) {
 #pragma unroll
-              for (int j = 0; j < 32; ++j) pk[b * 32 + j] = __float_as_uint(alpha * __uint_as_float(v[j]));
+              for (int j = 0; j < 64; ++j) pk[b * 64 + j] = __float_as_uint(alpha * __uint_as_float(v[j]));
             } else {
 #pragma unroll
-              for (int j = 0; j < 16; ++j) {
-                float a0 = alpha * __uint_as_float(v[2 * j]), a1 = alpha * __uint_as_float(v[2 * j + 1]);
-                if (pre_c) {
-                  const float2 cf = __half22float2(*reinterpret_cast<const __half2 *>(&cw[b * 16 + j]));
-                  a0 = fmaf(beta, cf.x, a0);
-                  a1 = fmaf(beta, cf.y, a1);
-                }
-                pk[b * 16 + j] = pack_half2(a0, a1);
-              }
+              for (int j = 0; j < 32; ++j)
+                pk[b * 32 + j] = pack_half2(alpha * __uint_as_float(v[2 * j]), alpha * __uint_as_float(v[2 * j + 1]));
             }
           }
           if (warp == 2 && lane == 0) HG_TRACE(it, 10 + h);
@@ -731,9 +742,6 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
             if constexpr (CG == 2) mbar_arrive_cluster_relaxed(tempty_addr + (buf * NH + h) * 8);
             else mbar_arrive_relaxed(&tempty[buf * NH + h]);
             if (warp == 2) HG_TRACE(it, 2 + h);
-          }
-          if constexpr (!OUT_F32) {
-            if (pre_c && h + 1 < NH) load_c_words<EPI_COLS_W>(p, cw, row, tn * BN + (h + 1) * UMMA_N + cgrp * EPI_COLS_W);
           }
 #pragma unroll
           for (int c = 0; c < EPI_COLS_W / EPI_COLS; ++c)

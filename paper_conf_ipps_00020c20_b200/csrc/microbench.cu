@@ -174,6 +174,52 @@ __global__ void __launch_bounds__(32, 1) tma_load_kernel(const __grid_constant__
 #endif
 }
 
+// Streaming pattern study for HBM-bound GEMM operands: each CTA owns bands of
+// `box_rows` rows of a [rows x row_len] FP16 tensor (row pitch row_len*2 B) and
+// reads them in 128-B-wide boxes with `depth` boxes in flight.
+//   order 0: GEMM order -- walk the k (column) boxes of a band, then the next band
+//   order 1: contiguous order -- the band's boxes column-major in memory order
+//            only when row_len == 64 (one box per row band); else same as 0
+__global__ void __launch_bounds__(32, 1) tma_stream_kernel(const __grid_constant__ CUtensorMap tm, int row_len,
+                                                            int rows, int box_rows, int depth,
+                                                            unsigned long long *out) {
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  uint8_t *smem = smem_raw + ((1024u - (raw & 1023u)) & 1023u);
+  const uint32_t box_bytes = static_cast<uint32_t>(box_rows) * 128u;
+  uint64_t *full = reinterpret_cast<uint64_t *>(smem + depth * box_bytes);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < depth; ++s) mbar_init(&full[s], 1);
+    fence_mbarrier_init();
+  }
+  __syncwarp();
+  if (threadIdx.x == 0) {
+    const int kboxes = row_len / 64;
+    const int bands = rows / box_rows;
+    const int my_bands = (bands - static_cast<int>(blockIdx.x) + static_cast<int>(gridDim.x) - 1) / static_cast<int>(gridDim.x);
+    const int total = my_bands * kboxes;
+    long long t0 = clock64();
+    uint32_t phase = 0;
+    for (int i = 0; i < total + depth; ++i) {
+      const int s = i % depth;
+      if (i >= depth) {
+        mbar_wait(&full[s], phase);
+        if (s == depth - 1) phase ^= 1u;
+      }
+      if (i < total) {
+        const int band = static_cast<int>(blockIdx.x) + (i / kboxes) * static_cast<int>(gridDim.x);
+        const int col = (i % kboxes) * 64;
+        mbar_arrive_expect_tx(&full[s], box_bytes);
+        tma_load_2d(&tm, smem_u32(smem + s * box_bytes), smem_u32(&full[s]), col, band * box_rows, 0);
+      }
+    }
+    long long t1 = clock64();
+    out[blockIdx.x] = static_cast<unsigned long long>(t1 - t0);
+  }
+#endif
+}
+
 }  // namespace mb
 
 namespace {
@@ -250,3 +296,24 @@ int mb_tma_load(const void *tensor, int rows, int iters, int grid, int streaming
 }
 
 }  // extern "C"
+
+// Streaming pattern study (see tma_stream_kernel); returns 0 on success.
+extern "C" int mb_tma_stream(const void *tensor, int row_len, int rows, int box_rows, int depth, int grid,
+                             unsigned long long *cycles_dev) {
+  EncodeTiledFn fn = encode_fn();
+  if (!fn) return 3;
+  CUtensorMap tm;
+  cuuint64_t dims[2] = {static_cast<cuuint64_t>(row_len), static_cast<cuuint64_t>(rows)};
+  cuuint64_t strides[1] = {static_cast<cuuint64_t>(row_len) * 2};
+  cuuint32_t box[2] = {64, static_cast<cuuint32_t>(box_rows)};
+  cuuint32_t estr[2] = {1, 1};
+  if (fn(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(tensor), dims, strides, box, estr,
+         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return 2;
+  const int smem = depth * box_rows * 128 + 1024 + 1024;
+  if (cudaFuncSetAttribute(mb::tma_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
+    return 1;
+  mb::tma_stream_kernel<<<grid, 32, smem>>>(tm, row_len, rows, box_rows, depth, cycles_dev);
+  return cudaGetLastError() == cudaSuccess ? 0 : 1;
+}

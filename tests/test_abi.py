@@ -56,6 +56,12 @@ def test_set_config_validation():
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(2, 128, 8, 0))) == 0
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(2, 128, 0, 0, 0, 3))) == 1   # stream_k 0..2
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 256, 0, 0, 0, 2))) == 0
+    # HBM-streaming kernel: chunk width a multiple of 16 in [16, 256] (0 = auto)
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(5, 112, 0, 0))) == 0
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(5, 0, 0, 0))) == 0
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(5, 100, 0, 0))) == 1
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(5, 272, 0, 0))) == 1
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(6, 0, 0, 0))) == 1
     assert lib.hgemm_set_config(None) == 0
 
 

@@ -126,6 +126,31 @@ def test_alpha_beta_integer(oracle_mod, kernel, bn, alpha, beta, out):
     assert np.array_equal(case.view(got).astype(np.float64), r)
 
 
+# (kernel, block_n, max_ctas): few persistent clusters, so every CTA runs several
+# tiles in a row and the staging boxes that carry C (TMA-loaded, combined in place,
+# TMA-stored) rotate across tiles and accumulator halves.
+BETA_CASES = [("tc2", 512, 4), ("tc2", 256, 4), ("tc1", 256, 3), ("tc1", 128, 5), ("tc2", 512, 0), ("tc1", 128, 0)]
+
+
+@pytest.mark.parametrize("kernel,bn,max_ctas", BETA_CASES)
+@pytest.mark.parametrize("tA,tB", [("T", "N"), ("N", "T")])
+@pytest.mark.parametrize("out", ["f16", "f32"])
+@pytest.mark.parametrize("m", [600, 597])   # 597: N (= m) not a multiple of 16 B -> chunked path
+def test_beta_random_multi_tile(oracle_mod, kernel, bn, max_ctas, tA, tB, out, m):
+    """beta != 0 on random inputs, several tiles per CTA, ragged m/n/k, ld padding."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config(kernel, block_n=bn, max_ctas=max_ctas, stream_k=1)
+    n, k = 1100, 200
+    C = inputs.uniform_f16(m, n, 17).astype(np.float32 if out == "f32" else np.float16)
+    case = GpuCase(inputs.uniform_f16(m, k, 15), inputs.uniform_f16(k, n, 16), tA, tB, 0.75, -1.25, C=C,
+                   out=out, pad=(8, 16, 8))
+    got = case.run_gpu()
+    _expect_kernel(case, kernel, bn)
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, got, r, ab)
+    assert np.all(np.isnan(case.padding(got).astype(np.float32)))
+
+
 @pytest.mark.parametrize("kernel,bn", KERNELS)
 @pytest.mark.parametrize("out", ["f16", "f32"])
 def test_beta_zero_never_reads_C(oracle_mod, kernel, bn, out):
@@ -366,3 +391,65 @@ def test_hgemm_host_buffers(oracle_mod, tA, tB, out, beta):
     # the host padding rows of C are untouched
     pad = case.padding(got).astype(np.float32)
     assert np.all(np.isnan(pad))
+
+
+# ------------------------------------------------------------------ HBM-streaming kernel (skinny, TN)
+@pytest.mark.parametrize("n", [64, 100, 128, 200, 256])
+@pytest.mark.parametrize("cw,max_ctas", [(48, 0), (112, 3), (16, 5), (128, 0)])
+@pytest.mark.parametrize("out,beta", [("f16", 0.0), ("f16", 0.5), ("f32", 0.0), ("f32", -1.5)])
+def test_stream_kernel(oracle_mod, n, cw, max_ctas, out, beta):
+    """Streaming kernel: chunks of cw rows of op(A) per persistent CTA (max_ctas
+    forces several chunks per CTA -> both TMEM accumulator buffers), 1 or 2
+    M-subtiles (n <= 128 / <= 256), ragged m, n and k, ld padding untouched."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("stream", block_n=cw, max_ctas=max_ctas)
+    m, k = 1003, 330
+    C = inputs.uniform_f16(m, n, 27).astype(np.float32 if out == "f32" else np.float16)
+    case = GpuCase(inputs.uniform_f16(m, k, 25), inputs.uniform_f16(k, n, 26), "T", "N", 1.25, beta, C=C,
+                   out=out, pad=(8, 16, 8))
+    got = case.run_gpu()
+    assert case.stats["last_kernel"] == "stream", case.stats
+    assert case.stats["block_n"] == (min(cw, 128) if n > 128 else cw), case.stats
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, got, r, ab)
+    if out == "f32":
+        rel = np.max(np.abs(case.view(got).astype(np.float64) - r) / np.maximum(ab + np.abs(beta) * np.abs(case.Cmat), 1e-30))
+        assert rel < 1e-5, rel
+    assert np.all(np.isnan(case.padding(got).astype(np.float32)))
+
+
+@pytest.mark.parametrize("n", [64, 256])
+def test_stream_kernel_integer_exact(oracle_mod, n):
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("stream", block_n=64)
+    opA = inputs.integer_f16(2000, 1024, 31, -4, 4)
+    opB = inputs.integer_f16(1024, n, 32, -4, 4)
+    case = GpuCase(opA, opB, "T", "N", out="f32")
+    got = case.view(case.run_gpu())
+    assert case.stats["last_kernel"] == "stream", case.stats
+    _, r, _ = case.oracle(oracle_mod)
+    assert np.array_equal(got.astype(np.float64), r)
+    a, b, expect = inputs.accumulator_width_case(2000, n, 4096)
+    case = GpuCase(a, b, "T", "N", out="f32")
+    assert np.all(case.view(case.run_gpu()) == expect)
+    assert case.stats["last_kernel"] == "stream", case.stats
+
+
+def test_stream_kernel_auto_and_fallback(oracle_mod):
+    """Automatic choice: the skinny TN shape of BJ configs[3] takes the streaming
+    kernel; the same shape in NN layout takes the tile kernels (still correct)."""
+    m, n, k = 16384, 64, 512
+    for tA, tB, expect in (("T", "N", "stream"), ("N", "N", None)):
+        case = GpuCase(inputs.uniform_f16(m, k, 41), inputs.uniform_f16(k, n, 42), tA, tB, out="f16")
+        got = case.run_gpu()
+        if expect:
+            assert case.stats["last_kernel"] == expect, case.stats
+        else:
+            assert case.stats["last_kernel"] != "stream", case.stats
+        rows = np.arange(0, m, 97)
+        cols = np.arange(n)
+        ii, jj = np.meshgrid(rows, cols, indexing="ij")
+        _, r, ab = oracle_mod.hgemm_ref_entries(m, n, k, 1.0, case.A, case.lda, case.B, case.ldb, 0.0, None,
+                                                case.ldc, tA, tB, "f16", ii.ravel(), jj.ravel())
+        g = case.view(got)[ii.ravel(), jj.ravel()].astype(np.float64)
+        assert np.all(np.abs(g - r) <= 1e-3 * ab + ulp16(np.maximum(np.abs(g), np.abs(r))))
