@@ -586,7 +586,10 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     int cw = cfg.kernel == HGEMM_KERNEL_STREAM && cfg.block_n ? cfg.block_n : stream_chunk(N, mt, di.num_sms);
     if (mt == 2 && cw > 128) cw = 128;
     CUtensorMap ta, tb;
-    bool ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
+    // Ak TMA box rows (hgemm_stream.cuh): 64 when M <= 64 and the stage's Bk part
+    // covers the 8 KB the M = 128 MMA reads past the 64 real Ak rows
+    const uint32_t a_rows = (M <= 64 && cw >= 64) ? 64u : 128u;
+    bool ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, a_rows);
     if (ok) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, cw);
     if (!ok) return HGEMM_ERR_CUDA;
     hg::StreamParams p = {};
@@ -596,9 +599,11 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     p.cw = cw;
     p.num_chunks = static_cast<int32_t>(cdiv(N, cw));
     p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
-    p.stage_bytes = static_cast<uint32_t>(mt) * 16384u + static_cast<uint32_t>(cw) * 128u;
+    p.a_bytes = a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u;
+    p.stage_bytes = p.a_bytes + static_cast<uint32_t>(cw) * 128u;
     p.stages = static_cast<int32_t>(std::min<uint32_t>(hg::kStreamMaxStages,
                                                        (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
+    p.probe = g_probe.load(std::memory_order_relaxed);
     p.k_rot = 1;
     if (const char *e = std::getenv("HGEMM_STREAM_ROT")) p.k_rot = std::atoi(e);  // experiments
     p.alpha = alpha;

@@ -331,6 +331,7 @@ __global__ void __launch_bounds__(192, 1)
 
   if (threadIdx.x == 64) SK_TRACE(6);
   // peers must not exit while their shared memory is being read
+  __syncwarp();  // reconverge the single-lane roles before the .aligned cluster barrier
   cluster_sync();
   if (threadIdx.x == 0) SK_TRACE(7);
   if (warp == 1) {

@@ -12,8 +12,9 @@
 //     multiple of the SM count -- every SM streams the same number of Bk rows
 //     (tiles of 128/256 columns would leave 20 of 148 SMs idle at m = 16384);
 //   * the ring depth is a runtime value: as many stages of (Ak 128 x 64 per
-//     M-subtile, L2-resident) + (Bk CW x 64, from HBM) as fit in 227 KB, so
-//     each SM keeps ~100 KB of Bk loads in flight (Little's law at ~7 TB/s);
+//     M-subtile, or 64 x 64 when M <= 64; L2-resident) + (Bk CW x 64, from
+//     HBM) as fit in 227 KB, so each SM keeps 100-140 KB of Bk loads in flight
+//     (Little's law; tools/stream_study.py measures the TMA streaming curve);
 //   * MT = M-subtiles of 128 rows (M <= 128: 1, M <= 256: 2); one tcgen05.mma
 //     M = 128, N = CW per subtile and K = 16 step (instruction descriptor N is
 //     a runtime field); accumulators double-buffered in TMEM across chunks;
@@ -37,12 +38,25 @@ struct StreamParams {
   int32_t num_chunks;     // ceil(N / cw)
   int32_t num_k_blocks;   // ceil(K / 64)
   int32_t stages;         // ring depth (<= kStreamMaxStages)
-  uint32_t stage_bytes;   // MT * 16 KB + cw * 128, a multiple of 1024
+  uint32_t stage_bytes;   // a_bytes + cw * 128, a multiple of 1024
+  uint32_t a_bytes;       // Ak bytes per stage: MT * 16 KB, or 8 KB when M <= 64 (see below)
   int32_t k_rot;          // 1: CTA c walks its k-blocks starting at c * nkb / gridDim (see below)
   float alpha, beta;
   void *D;
   int64_t ldd;
+  unsigned long long *probe;  // HGEMM_TRACE builds: per-CTA %globaltimer events (tools/trace_stream.py)
 };
+
+#ifdef HGEMM_TRACE
+#define ST_TRACE(f)                                                                                  \
+  do {                                                                                               \
+    if (p.probe != nullptr) p.probe[8 * blockIdx.x + (f)] = globaltimer_ns();                        \
+  } while (0)
+#else
+#define ST_TRACE(f) \
+  do {              \
+  } while (0)
+#endif
 
 constexpr int kStreamMaxStages = 16;
 constexpr uint32_t kStreamSmemBytes = 227u * 1024u;
@@ -67,6 +81,11 @@ __global__ void __launch_bounds__(192, 1)
                         const StreamParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
   constexpr uint32_t A_SUB = 128u * 64u * 2u;  // one 128-row Ak subtile of a k-block (16 KB)
+  // M <= 64: the TMA box holds the 64 real Ak rows only (8 KB) and Bk follows
+  // at +8 KB; the M = 128 MMA then reads Bk bytes as Ak rows 64..127, which
+  // only feed accumulator lanes 64..127 -- rows >= M that are never stored.
+  // One stage shrinks from 30 to 22 KB, so the ring holds 10 instead of 7.
+  const uint32_t a_bytes = p.a_bytes;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw_u32 = smem_u32(smem_raw);
   uint8_t *smem = smem_raw + ((1024u - (raw_u32 & 1023u)) & 1023u);
@@ -80,6 +99,7 @@ __global__ void __launch_bounds__(192, 1)
 
   const uint32_t warp = warp_id();
   const uint32_t lane = lane_id();
+  if (threadIdx.x == 0) ST_TRACE(0);
   const int cw = p.cw;
   // k-block order: with k_rot, CTA c starts its k loop at c * nkb / gridDim and
   // wraps, so that at any moment the CTAs read different column offsets of
@@ -110,6 +130,7 @@ __global__ void __launch_bounds__(192, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (threadIdx.x == 0) ST_TRACE(1);
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer
@@ -125,7 +146,7 @@ __global__ void __launch_bounds__(192, 1)
           const uint32_t fb = smem_u32(&full[stage]);
 #pragma unroll
           for (int t = 0; t < MT; ++t) tma_load_2d(&tmA, sa + t * A_SUB, fb, kb * 64, t * 128, 0);
-          tma_load_2d(&tmB, sa + MT * A_SUB, fb, kb * 64, n0, 0);
+          tma_load_2d(&tmB, sa + a_bytes, fb, kb * 64, n0, 0);
           if (++stage == static_cast<uint32_t>(stages)) { stage = 0; phase ^= 1u; }
         }
       }
@@ -145,8 +166,9 @@ __global__ void __launch_bounds__(192, 1)
         for (int kb = 0; kb < nkb; ++kb) {  // iteration index (the smem stage holds k-block (kb + kb_rot) % nkb)
           mbar_wait(&full[stage], phase);
           tc_fence_after();
+          if (it == 0 && kb == 0) ST_TRACE(2);
           const uint32_t sa = smem_u32(smem + stage * stage_bytes);
-          const uint32_t sb = sa + MT * A_SUB;
+          const uint32_t sb = sa + a_bytes;
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
             const uint64_t bd = sdesc_k_sw128(sb + k * 32);
@@ -159,6 +181,7 @@ __global__ void __launch_bounds__(192, 1)
           if (++stage == static_cast<uint32_t>(stages)) { stage = 0; phase ^= 1u; }
         }
         umma_commit<1>(&tfull[buf]);
+        if (it == 0) ST_TRACE(3);
       }
     }
   } else {
@@ -172,6 +195,7 @@ __global__ void __launch_bounds__(192, 1)
       if (lane == 0) mbar_wait(&tfull[buf], acc_phase);
       __syncwarp();
       tc_fence_after();
+      if (warp == 2 && lane == 0 && it == 0) ST_TRACE(4);
       const int n0 = ch * cw;
 #pragma unroll
       for (int t = 0; t < MT; ++t) {
@@ -244,11 +268,14 @@ __global__ void __launch_bounds__(192, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tempty[buf]);
+      if (warp == 2 && lane == 0 && it == 0) ST_TRACE(5);
     }
   }
 
+  __syncwarp();  // reconverge the single-lane roles before the .aligned CTA barrier
   tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0) ST_TRACE(6);
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc<1>(tmem_base, 512);

@@ -905,6 +905,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     if (lane == 0) bulk_wait_group<0>();
   }
 
+  // Reconverge each warp (the role code ran on one lane of warps 0/1) before the
+  // CTA barrier: bar.sync is .aligned, a partially arrived warp must not be able to
+  // release it while the epilogue still reads TMEM.
+  __syncwarp();
   tc_fence_before();
   __syncthreads();
   if (p.probe != nullptr && blockIdx.x == 0 && threadIdx.x == 0) {

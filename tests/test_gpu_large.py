@@ -76,7 +76,7 @@ def test_metric_config_8192(oracle_mod, tA, tB, out):
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("name", ["cfg1_256_NN_f32", "cfg3_bert_ffn1_4096", "cfg3_bert_ffn2_4096",
+@pytest.mark.parametrize("name", ["cfg1_256_NN_f32", "cfg3_bert_ffn1_4096", "cfg3_bert_ffn1_16384", "cfg3_bert_ffn2_4096",
                                   "cfg3_lstm_b64", "cfg3_lstm_b256", "cfg3_lstm_b1024", "cfg4_skinny_n64",
                                   "cfg4_skinny_n128", "cfg4_skinny_n256"])
 def test_baseline_configs(oracle_mod, name):
