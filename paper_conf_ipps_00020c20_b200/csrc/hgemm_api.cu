@@ -206,12 +206,12 @@ bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags)
 }
 
 // ----------------------------------------------------------------- TC launch
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32>
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC>
 hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &td, const TcParams &p0,
                          int dev, const DeviceInfo &di, int max_ctas, int sk_mode, bool *sk_used,
                          cudaStream_t stream) {
   using S = TcShape<BN, CG, OUT_F32>;
-  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32>;
+  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC>;
   static int attr_done[kMaxDevices] = {};
   static int max_clusters[kMaxDevices] = {};
   if (!attr_done[dev]) {
@@ -219,18 +219,18 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
       return HGEMM_ERR_CUDA;
     if (CG == 2) {
       cudaLaunchConfig_t qc = {};
-      qc.gridDim = dim3(2 * (di.num_sms / 2));
+      qc.gridDim = dim3(CG * MC * (di.num_sms / (CG * MC)));
       qc.blockDim = dim3(S::THREADS);
       qc.dynamicSmemBytes = S::SMEM_BYTES;
       cudaLaunchAttribute qa[1];
       qa[0].id = cudaLaunchAttributeClusterDimension;
-      qa[0].val.clusterDim.x = 2;
+      qa[0].val.clusterDim.x = CG * MC;
       qa[0].val.clusterDim.y = 1;
       qa[0].val.clusterDim.z = 1;
       qc.attrs = qa;
       qc.numAttrs = 1;
       int n = 0;
-      if (cudaOccupancyMaxActiveClusters(&n, kern, &qc) != cudaSuccess || n <= 0) n = di.num_sms / 2;
+      if (cudaOccupancyMaxActiveClusters(&n, kern, &qc) != cudaSuccess || n <= 0) n = di.num_sms / (CG * MC);
       max_clusters[dev] = n;
     } else {
       max_clusters[dev] = di.num_sms;
@@ -239,7 +239,7 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   }
   const int tiles = p0.num_m_tiles * p0.num_n_tiles;
   int units = max_clusters[dev];
-  if (max_ctas > 0) units = std::max(1, std::min(units, max_ctas / CG));
+  if (max_ctas > 0) units = std::max(1, std::min(units, max_ctas / (CG * MC)));
   int clusters = std::min(tiles, units);
   TcParams p = p0;
   p.dp_tiles = tiles;
@@ -247,11 +247,11 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   p.sk_ws = nullptr;
   p.sk_flags = nullptr;
   *sk_used = false;
-  if (S::NH == 1) {
+  if (S::NH == 1 && MC == 1) {
     const int dp = sk_plan(tiles, units, p.num_k_blocks, sk_mode);
     float *ws = nullptr;
     int *flags = nullptr;
-    if (dp >= 0 && units * CG <= di.num_sms && sk_workspace(dev, stream, di.num_sms, &ws, &flags)) {
+    if (dp >= 0 && units * CG * MC <= di.num_sms && sk_workspace(dev, stream, di.num_sms, &ws, &flags)) {
       p.dp_tiles = dp;
       p.sk_u0 = static_cast<int64_t>(dp) * p.num_k_blocks;
       p.sk_units = static_cast<int64_t>(tiles - dp) * p.num_k_blocks;
@@ -262,13 +262,13 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
     }
   }
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(clusters * CG);
+  cfg.gridDim = dim3(clusters * CG * MC);
   cfg.blockDim = dim3(S::THREADS);
   cfg.dynamicSmemBytes = S::SMEM_BYTES;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = CG;
+  attr[0].val.clusterDim.x = CG * MC;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
@@ -278,13 +278,13 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   return HGEMM_SUCCESS;
 }
 
-template <int BN, int CG>
+template <int BN, int CG, int MC = 1>
 hgemm_status_t dispatch_tc_layout(bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
                                   const CUtensorMap &td, const TcParams &p, int dev, const DeviceInfo &di,
                                   int max_ctas, int sk_mode, bool *sk_used, cudaStream_t s) {
 #define HG_CASE(AM, BM_, F)                                                               \
   if (a_mn == AM && b_mn == BM_ && f32 == F)                                              \
-    return launch_tc<BN, CG, AM, BM_, F>(ta, tb, td, p, dev, di, max_ctas, sk_mode, sk_used, s);
+    return launch_tc<BN, CG, AM, BM_, F, MC>(ta, tb, td, p, dev, di, max_ctas, sk_mode, sk_used, s);
   HG_CASE(false, false, false)
   HG_CASE(false, false, true)
   HG_CASE(false, true, false)
@@ -672,13 +672,22 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   if (forced_cg && cfg.block_n) { cg = forced_cg; bn = cfg.block_n; }
   else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, cfg.stream_k, cg, bn);
   const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
+  // MC = 2: two CTA pairs per cluster share (multicast) the Bk half-boxes
+  // (measured slower everywhere: a 4-CTA cluster strands SMs of the GPCs and couples
+  // the two pairs' pipelines; built only with -DHGEMM_ENABLE_MC)
+  int mc = 1;
+#ifdef HGEMM_ENABLE_MC
+  if (cg == 2) {
+    if (const char *e = std::getenv("HGEMM_MC")) mc = std::atoi(e) == 2 ? 2 : 1;  // experiments
+  }
+#endif
 
   CUtensorMap ta, tb;
   bool ok;
   if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
   else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
   if (ok) {
-    if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, b_rows);
+    if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, b_rows / mc);
     else ok = make_map(&tb, A, static_cast<uint64_t>(m), static_cast<uint64_t>(k), lda, 64, 64);
   }
   // D = C^T row-major (N = m contiguous), stored in 32-row x 128-B swizzled boxes
@@ -690,10 +699,10 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   p.M = static_cast<int32_t>(M);
   p.N = static_cast<int32_t>(N);
   p.K = static_cast<int32_t>(k);
-  p.num_m_tiles = static_cast<int32_t>(cdiv(M, 128 * cg));
+  p.num_m_tiles = static_cast<int32_t>(cdiv(M, 128 * cg * mc));
   p.num_n_tiles = static_cast<int32_t>(cdiv(N, bn));
   p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
-  p.group_m = cfg.group_m > 0 ? cfg.group_m : 16;  // measured best with 256x512 pair tiles (profiles/)
+  p.group_m = cfg.group_m > 0 ? cfg.group_m : 16 / mc;  // measured best with 256x512 pair tiles (profiles/)
   p.group_m = std::max(1, std::min(p.group_m, p.num_m_tiles));
   if (const char *e = std::getenv("HGEMM_GROUP_N")) {  // experiments: group along N instead
     const int gn = std::atoi(e);
@@ -712,6 +721,13 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   hgemm_status_t st;
   bool sk_used = false;
   const int skm = cfg.stream_k;
+#ifdef HGEMM_ENABLE_MC
+  if (cg == 2 && bn == 512 && mc == 2)
+    st = dispatch_tc_layout<512, 2, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
+  else if (cg == 2 && mc == 2)
+    st = dispatch_tc_layout<256, 2, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
+  else
+#endif
   if (cg == 2 && bn == 512)
     st = dispatch_tc_layout<512, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
   else if (cg == 2)

@@ -173,15 +173,15 @@ struct TcShape {
   static constexpr int EPI_COLS = OUT_F32 ? 32 : 64;   // one 128-B staging row per thread
   // 8 epilogue warps: two per TMEM lane quadrant, each owning half of every
   // accumulator half's columns.  Each warp stages 32 x 128-B boxes in EPI_BUFS
-  // buffers; two buffers when that still leaves >= 4 ring stages.
+  // buffers.  One buffer: the 32 KB it frees buys one more ring stage, which
+  // measured faster than a second staging box everywhere (BERT-FFN1 with
+  // beta = 1 and 256-wide tiles: 5 -> 6 stages, +6%).
   static constexpr int EPI_WARPS = 8;
   static constexpr int EPI_COLS_W = UMMA_N / 2;        // columns per warp per accumulator half
-  static constexpr int RING_FIT2 =
-      static_cast<int>((227u * 1024u - EPI_WARPS * 2u * 4096u - 2048u) / STAGE_BYTES);
 #ifdef HGEMM_EPI_BUFS
   static constexpr int EPI_BUFS = HGEMM_EPI_BUFS;
 #else
-  static constexpr int EPI_BUFS = RING_FIT2 >= 4 ? 2 : 1;
+  static constexpr int EPI_BUFS = 1;
 #endif
   static constexpr uint32_t EPI_BYTES = EPI_WARPS * EPI_BUFS * 32 * 128;
   // As many ring stages as fit in 227 KB next to the staging buffers, barriers and alignment slack.
@@ -275,7 +275,14 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
   } while (0)
 #endif
 
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32>
+// MC = 2 (CG = 2 only): a cluster of two CTA pairs computes two vertically
+// adjacent pair tiles (rows tm*2*256 .. +512) over the same Bk columns; each
+// Bk half-box is loaded once, half by each pair, and multicast to the CTA at the
+// same position in both pairs, so the L2 -> SM operand traffic per CTA drops
+// from (16 + 2*16) KB to (16 + 16) KB per k-block for BN = 512 (DESIGN.md
+// "Multicast").  A stage may be overwritten only after both pairs' MMAs have
+// read it: empty[] counts MC arrivals, multicast by each pair's MMA leader.
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC = 1>
 __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     hgemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmD, const TcParams p) {
@@ -312,9 +319,17 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
 
   const uint32_t warp = warp_id();
   const uint32_t lane = lane_id();
-  const uint32_t rank = (CG == 2) ? cluster_ctarank() : 0u;
-  const int cluster_id = static_cast<int>(blockIdx.x) / CG;
-  const int num_clusters = static_cast<int>(gridDim.x) / CG;
+  static_assert(MC == 1 || (MC == 2 && CG == 2), "multicast needs CTA pairs");
+  const uint32_t rank = (CG == 2) ? cluster_ctarank() : 0u;  // in the cluster (0 .. CG*MC-1)
+  const uint32_t prank = rank & (CG - 1u);                    // in the CTA pair
+  const uint32_t pair = rank / CG;                            // pair in the cluster (MC = 2)
+  const uint32_t leader = rank - prank;                       // rank of this pair's MMA leader
+  const int cluster_id = static_cast<int>(blockIdx.x) / (CG * MC);
+  const int num_clusters = static_cast<int>(gridDim.x) / (CG * MC);
+  // multicast masks of the MMA leader's commits: its own pair (tmem_full), and
+  // every CTA whose smem stages it read (empty)
+  const uint16_t pair_mask = static_cast<uint16_t>(((1u << CG) - 1u) << leader);
+  const uint16_t empty_mask = static_cast<uint16_t>(MC == 2 ? 0xFu : pair_mask);
   
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
@@ -325,7 +340,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     if (lane == 0) {
       for (int s = 0; s < STAGES; ++s) {
         mbar_init(&full[s], 1);
-        mbar_init(&empty[s], 1);
+        mbar_init(&empty[s], MC);
       }
       for (int a = 0; a < ACC; ++a) {
         for (int h = 0; h < NH; ++h) {
@@ -364,8 +379,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i) {
         int tm, tn;
         tile_coords(wi.tile, p, tm, tn);
-        const int a_row = tm * BM * CG + static_cast<int>(rank) * BM;
-        const int b_row0 = tn * BN + static_cast<int>(rank) * B_ROWS;
+        const int a_row = (tm * MC + static_cast<int>(pair)) * BM * CG + static_cast<int>(prank) * BM;
+        const int b_row0 = tn * BN + static_cast<int>(prank) * B_ROWS;
         for (int kb = wi.kb0; kb < wi.kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1u);
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
@@ -375,8 +390,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
             mbar_arrive_expect_tx(&full[stage], STAGE_BYTES);
             fb = smem_u32(&full[stage]);
           } else {
-            if (rank == 0) mbar_arrive_expect_tx(&full[stage], 2 * STAGE_BYTES);
-            fb = mapa_shared(smem_u32(&full[stage]), 0);
+            if (prank == 0) mbar_arrive_expect_tx(&full[stage], 2 * STAGE_BYTES);
+            fb = mapa_shared(smem_u32(&full[stage]), leader);
           }
           const int k0 = kb * BK;
           if constexpr (!A_MN) {
@@ -393,6 +408,16 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
           for (int h = 0; h < NH; ++h) {
             const uint32_t sbh = sb + h * B_HALF_BYTES;
             const int b_row = b_row0 + h * UMMA_N;
+            if constexpr (MC == 2) {
+              // this pair's share of the half-box, delivered to the same CTA position of both pairs
+              const uint16_t mc_mask = static_cast<uint16_t>((1u << prank) | (1u << (CG + prank)));
+              if constexpr (!B_MN)
+                tma_load_2d_pair_mc(&tmB, sbh + pair * (B_ROWS / 2) * 128u, fb, k0,
+                                    b_row + static_cast<int>(pair) * (B_ROWS / 2), mc_mask);
+              else
+                tma_load_2d_pair_mc(&tmB, sbh + pair * 8192u, fb, b_row + 64 * static_cast<int>(pair), k0, mc_mask);
+              continue;
+            }
             if constexpr (!B_MN) {
               if constexpr (CG == 1) tma_load_2d(&tmB, sbh, fb, k0, b_row, pol_b);
               else tma_load_2d_pair(&tmB, sbh, fb, k0, b_row, pol_b);
@@ -410,7 +435,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (leader CTA)
-    if (rank == 0 && lane == 0) {
+    if (prank == 0 && lane == 0) {
       // NH == 2 (one 512-column accumulator in two halves):
       //  * at a tile start, half 1 may still be draining: half-0 MMAs run up to
       //    MAX_LEAD k-blocks ahead (their smem stages stay resident) until
@@ -463,7 +488,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         auto flush_h1 = [&](int upto) {  // issue half 1 for k-blocks [kb1, upto)
           while (kb1 < upto) {
             issue_half(stage1, 1, kb1, d_tmem);
-            umma_commit<CG>(&empty[stage1]);  // both halves have consumed this stage
+            umma_commit_mask<CG>(&empty[stage1], empty_mask);  // both halves have consumed this stage
             if (++stage1 == STAGES) stage1 = 0;
             ++kb1;
           }
@@ -502,7 +527,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
                   umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
                 }
               }
-              umma_commit<CG>(&empty[stage]);
+              umma_commit_mask<CG>(&empty[stage], empty_mask);
               ++kb1;
               if (++stage1 == STAGES) stage1 = 0;
             } else {
@@ -512,17 +537,17 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
             }
           } else {
             issue_half(stage, 0, kb, d_tmem);
-            umma_commit<CG>(&empty[stage]);  // frees the smem stage once these MMAs retire
+            umma_commit_mask<CG>(&empty[stage], empty_mask);  // frees the smem stage once these MMAs retire
           }
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
         }
         if constexpr (NH == 2) {
-          umma_commit<CG>(&tfull[buf * NH + 0]);  // half 0 complete: the epilogue may drain it
+          umma_commit_mask<CG>(&tfull[buf * NH + 0], pair_mask);  // half 0 complete: the epilogue may drain it
           if (!h1_ready) acquire_h1(true);
           flush_h1(nkb);                            // the lagging half-1 k-blocks
-          umma_commit<CG>(&tfull[buf * NH + 1]);
+          umma_commit_mask<CG>(&tfull[buf * NH + 1], pair_mask);
         } else {
-          umma_commit<CG>(&tfull[buf]);             // accumulator ready for the epilogue
+          umma_commit_mask<CG>(&tfull[buf], pair_mask);  // accumulator ready for the epilogue
         }
         HG_TRACE(it, 0);
         HG_CTRACE(it, 0);
@@ -537,7 +562,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     const uint32_t ew = warp - 2u;                   // epilogue warp index 0..7
     const int cgrp = static_cast<int>(ew >> 2);      // which half of each accumulator half's columns
     const uint32_t stg = smem_u32(epi_smem) + ew * (EPI_BUFS * 32u * 128u);
-    const uint32_t tempty_addr = (CG == 2) ? mapa_shared(smem_u32(&tempty[0]), 0) : smem_u32(&tempty[0]);
+    const uint32_t tempty_addr = (CG == 2) ? mapa_shared(smem_u32(&tempty[0]), leader) : smem_u32(&tempty[0]);
     const float alpha = p.alpha, beta = p.beta;
     uint32_t nstore = 0;
     int it = 0;
@@ -584,7 +609,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
       };
       const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
       const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
-      const int row_base = tm * BM * CG + static_cast<int>(rank) * BM + static_cast<int>(quad) * 32;
+      const int row_base = (tm * MC + static_cast<int>(pair)) * BM * CG + static_cast<int>(prank) * BM +
+                           static_cast<int>(quad) * 32;
       const int row = row_base + static_cast<int>(lane);
       // beta != 0 (whole tiles, N a multiple of 16 B): C is brought into this warp's
       // staging boxes by TMA before the accumulator is ready, combined in place and

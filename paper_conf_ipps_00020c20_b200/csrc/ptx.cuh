@@ -167,6 +167,17 @@ __device__ __forceinline__ void tma_load_2d_pair(const CUtensorMap *m, uint32_t 
       "l"(reinterpret_cast<uint64_t>(m)), "r"(bar_cluster), "r"(c0), "r"(c1), "l"(policy)
       : "memory");
 }
+// CTA-pair tile load multicast to the CTAs in `mask` (same smem offset in each);
+// each destination's bytes complete on the barrier at `bar_cluster`'s offset in
+// that destination's pair leader (the peer bit of the address is cleared).
+__device__ __forceinline__ void tma_load_2d_pair_mc(const CUtensorMap *m, uint32_t dst, uint32_t bar_cluster,
+                                                    int32_t c0, int32_t c1, uint16_t mask) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster"
+      " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(bar_cluster & 0xFEFFFFFFu), "r"(c0), "r"(c1), "h"(mask)
+      : "memory");
+}
 __device__ __forceinline__ uint64_t l2_policy_evict_last() {
   uint64_t p;
   asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
@@ -305,6 +316,20 @@ __device__ __forceinline__ void umma_commit(uint64_t *bar) {
                  : "memory");
   } else {
     const uint16_t mask = 0x3;
+    asm volatile(
+        "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+            smem_u32(bar)),
+        "h"(mask)
+        : "memory");
+  }
+}
+
+// As umma_commit, with an explicit multicast mask of cluster CTAs (CG == 2).
+template <int CG>
+__device__ __forceinline__ void umma_commit_mask(uint64_t *bar, uint16_t mask) {
+  if constexpr (CG == 1) {
+    umma_commit<1>(bar);
+  } else {
     asm volatile(
         "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
             smem_u32(bar)),
