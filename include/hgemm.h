@@ -118,7 +118,7 @@ typedef struct {
     int32_t group_m;   /* L2 raster group height in tiles (0 = auto) */
     int32_t max_ctas;  /* cap on persistent CTAs (0 = all SMs) */
     int32_t splits;    /* HGEMM_KERNEL_SPLITK: K splits per tile, 2, 4 or 8 (0 = auto) */
-    int32_t stream_k;  /* tensor-core kernels with block_n <= 256: 0 = auto, 1 = never, 2 = whenever the
+    int32_t stream_k;  /* tensor-core tile kernels: 0 = auto, 1 = never, 2 = whenever the
                           tile count is not a multiple of the persistent cluster count.  Stream-K cuts
                           the k-blocks of the last tiles into equal contiguous ranges, one per cluster;
                           a tile split between clusters is summed in k order through a library-owned

@@ -167,7 +167,7 @@ int sk_plan(int64_t tiles, int64_t units, int64_t nkb, int mode) {
 }
 
 // Library-owned FP32 partial slots + flags, one set per (device, stream):
-// room for one 128 x 256 FP32 slot and one flag per SM.  Flags are zero
+// room for one 128 x 512 FP32 slot and one flag per SM.  Flags are zero
 // between launches (every consumer resets the flag it waited for).
 struct SkWorkspace {
   int dev;
@@ -192,7 +192,7 @@ bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags)
   if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) return false;
   float *w = nullptr;
   int *f = nullptr;
-  if (cudaMalloc(&w, static_cast<size_t>(num_sms) * 128 * 256 * sizeof(float)) != cudaSuccess) return false;
+  if (cudaMalloc(&w, static_cast<size_t>(num_sms) * 128 * 512 * sizeof(float)) != cudaSuccess) return false;
   if (cudaMalloc(&f, static_cast<size_t>(num_sms) * sizeof(int)) != cudaSuccess ||
       cudaMemsetAsync(f, 0, static_cast<size_t>(num_sms) * sizeof(int), s) != cudaSuccess) {
     cudaFree(w);
@@ -247,7 +247,7 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   p.sk_ws = nullptr;
   p.sk_flags = nullptr;
   *sk_used = false;
-  if (S::NH == 1 && MC == 1) {
+  if (MC == 1) {
     const int dp = sk_plan(tiles, units, p.num_k_blocks, sk_mode);
     float *ws = nullptr;
     int *flags = nullptr;
@@ -441,7 +441,9 @@ void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, 
     const int64_t units = num_sms / c.cg;
     double waves = static_cast<double>(cdiv(tiles, units));
     const int64_t nkb = cdiv(K, 64);
-    if (c.bn <= 256 && sk_plan(tiles, units, nkb, sk_mode) >= 0)  // stream-K: fractional waves
+    // stream-K: fractional waves (256-wide tiles only: with 512-wide tiles the FP32
+    // partials of a split tile are twice as large and it measured slower everywhere)
+    if (c.bn <= 256 && sk_plan(tiles, units, nkb, sk_mode) >= 0)
       waves = static_cast<double>(tiles) / units + sk_overhead_waves(nkb);
     const double t = waves * (128.0 * c.cg * c.bn) / (c.cg * eff);
     if (t < best * 0.999) { best = t; cg = c.cg; bn = c.bn; }

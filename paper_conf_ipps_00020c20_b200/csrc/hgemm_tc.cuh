@@ -571,10 +571,13 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
     constexpr int VEC = OUT_F32 ? 4 : 8;
     const bool fast = ((p.N & (VEC - 1)) == 0) && beta == 0.0f;
     constexpr int PKW = OUT_F32 ? EPI_COLS_W : EPI_COLS_W / 2;  // packed result words per thread per half
-    // Stream-K partial slots: per CTA slot, per epilogue warp, EPI_COLS_W/32 boxes of
+    // Stream-K partial slots: per CTA slot, per epilogue warp, NH*EPI_COLS_W/32 boxes of
     // 32 rows x 32 FP32 (4 KB, 16-B chunks swizzled like the staging boxes),
-    // written and read with 1-D bulk copies.
-    constexpr int SK_BOXES = EPI_COLS_W / 32;
+    // written and read with 1-D bulk copies.  Chunk index over both accumulator
+    // halves: h * NCH + c.  (Direct 16-B register<->global partial transfers were
+    // measured slower than this staged bulk path.)
+    constexpr int NCH = EPI_COLS_W / EPI_COLS;
+    constexpr int SK_BOXES = NH * EPI_COLS_W / 32;
     auto sk_box = [&](int slot_cluster, int j) -> uint8_t * {
       return reinterpret_cast<uint8_t *>(p.sk_ws) +
              ((static_cast<int64_t>(slot_cluster * CG + static_cast<int>(rank)) * S::EPI_WARPS + ew) * SK_BOXES + j) *
@@ -597,7 +600,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         while (c_hi < num_clusters && sk_begin(p, c_hi, num_clusters) < tile_end) ++c_hi;
       }
       const int n_contrib = c_hi - cluster_id - 1;
-      const int sk_seq = (EPI_COLS_W / EPI_COLS) * n_contrib;  // (chunk, contributor) loads, chunk-major
+      const int sk_seq = NH * NCH * n_contrib;  // (chunk, contributor) loads, chunk-major
       // bulk-load step s of the head's partial stream into staging buffer s & 1
       auto sk_issue = [&](int s) {
         const int c = s / n_contrib, q = s - c * n_contrib, b = s & 1;
@@ -818,7 +821,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
               fence_proxy_async_smem();
               __syncwarp();
               if (lane == 0) {
-                bulk_store_1d(sk_box(cluster_id, c * (EPI_COLS / 32) + x), sbuf, 4096);
+                bulk_store_1d(sk_box(cluster_id, (h * NCH + c) * (EPI_COLS / 32) + x), sbuf, 4096);
                 bulk_commit_group();
               }
               ++nstore;
@@ -826,7 +829,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
             continue;
           }
           for (int q = 0; q < n_contrib; ++q) {  // mode 2: add the later k segments, in k order
-            const int sidx = c * n_contrib + q, b = sidx & 1;
+            const int sidx = (h * NCH + c) * n_contrib + q, b = sidx & 1;
             mbar_wait(&skbar[ew * 2 + b], sk_uses[b] & 1u);
             ++sk_uses[b];
 #pragma unroll

@@ -116,3 +116,6 @@ STRONG_SCALING = {"cfg5_sharded_32768"}
 
 # Square sweep of the paper's evaluation: W = 1024..16384 step 256.
 SQUARE_SWEEP = list(range(1024, 16384 + 1, 256))
+# ... as bench workloads "sq_<W>" (BASELINE.json configs[1], paper layout TN, FP16 out)
+for _w in SQUARE_SWEEP:
+    WORKLOADS[f"sq_{_w}"] = (_w, _w, _w, "T", "N", 1.0, 0.0, "f16")

@@ -238,7 +238,7 @@ def test_all_kernels_agree_on_random(oracle_mod):
 # 40 / 24 k-blocks (two segments per split tile), 12 (three segments: tiles
 # fewer than clusters) and whole data-parallel waves before the stream-K part.
 SK_CASES = [("tc2", 256, 8), ("tc2", 256, 32), ("tc1", 256, 8), ("tc1", 128, 12), ("tc1", 128, 40),
-            ("tc1", 128, 4)]
+            ("tc1", 128, 4), ("tc2", 512, 8), ("tc2", 512, 4), ("tc2", 512, 12)]
 
 
 @pytest.mark.parametrize("kernel,bn,max_ctas", SK_CASES)

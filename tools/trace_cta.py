@@ -23,9 +23,10 @@ ap.add_argument("k", type=int)
 ap.add_argument("--beta", type=float, default=1.0)
 ap.add_argument("--kernel", default="auto")
 ap.add_argument("--bn", type=int, default=0)
+ap.add_argument("--sk", type=int, default=0)
 a = ap.parse_args()
 if a.kernel != "auto":
-    binding.set_config(a.kernel, block_n=a.bn)
+    binding.set_config(a.kernel, block_n=a.bn, stream_k=a.sk)
 m, n, k = a.m, a.n, a.k
 A = (torch.rand(m, k, device="cuda") * 2 - 1).half()
 B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
@@ -43,6 +44,8 @@ rows = [v[264 + 8 * b: 272 + 8 * b] for b in range(160) if v[264 + 8 * b]]
 t0 = min(r[0] for r in rows)
 names = ["start", "end", "i0_mma", "i0_wake", "i0_done", "i1_mma", "i1_wake", "i1_done"]
 print(f"{len(rows)} CTAs; kernel span {max(r[1] for r in rows) - t0} ns")
+for b, r in enumerate(rows[:6]):
+    print(f"cta {b:3d} " + " ".join(f"{nm}={(x - t0) if x else -1}" for nm, x in zip(names, r)))
 for f, nm in enumerate(names):
     xs = [r[f] - t0 for r in rows if r[f]]
     if xs:
