@@ -147,6 +147,84 @@ int64_t hgemm_launch_count(void);
  * (clk1-clk0)/(ns1-ns0) GHz.  NULL (the default) disables it.  Process-global. */
 hgemm_status_t hgemm_set_probe(unsigned long long *device_buf);
 
+/* ------------------------------------------------------------------------
+ * Sharded path: all-gather of op(A) fused with the GEMM
+ * (BASELINE.json north_star (3): "N-column slabs of B and C are sharded per
+ * GPU with A replicated"; the paper itself
+ * is single-GPU, its C = alpha*A*B + beta*C is P:47, SII-A).
+ *
+ * Rank q of `world` owns rows [row_splits[q], row_splits[q+1]) of op(A)
+ * (row_splits: host array of world+1 values, 0 = row_splits[0] <= ... <=
+ * row_splits[world] = m).  Every rank holds a full-size GATHER BUFFER `A`
+ * in the paper's layout, transA = 'T' (A stored k x m column-major, lda >= k,
+ * so row i of op(A) is the contiguous run A + i*lda of k FP16 values), in
+ * which its own rows are already written.  A_peers (host array of `world`
+ * device pointers) holds every other rank's gather buffer as mapped into this
+ * process (hgemm_ipc_open below; for ranks on one device, plain pointers);
+ * A_peers[rank] is ignored.  The caller must make the peers' own rows
+ * complete before the call (e.g. a barrier after writing them).
+ *
+ * ONE persistent tcgen05 kernel on `stream` does both steps: an extra copy
+ * warp in every CTA pulls the peers' rows of op(A) with 16-B loads from the
+ * P2P-mapped peer buffers (NVLink/NVSwitch) into `A`, in copy units of ~64 KB
+ * of rows taken from a shared work index in the order owners rank+1, rank+2,
+ * ... (mod world), and counts each finished unit in its chunk's counter; the
+ * TMA producer of each CTA waits, before the first load of a tile, until
+ * every chunk of op(A) rows the tile reads is complete (local chunks never
+ * wait), and tiles are scheduled chunk by chunk starting with the local rows,
+ * so the transfer overlaps the MMAs tile by tile.  Chunk c is rows
+ * [c*chunk_rows, (c+1)*chunk_rows) of op(A).  The result is C = alpha*op(A)*
+ * op(B) + beta*C (m x n, same meaning as hgemm() with transA = 'T'), bitwise
+ * identical to hgemm() on the gathered A, and `A` ends holding all m rows.
+ * `workspace`: caller-owned device memory of workspace_ints >= 1 +
+ * ceil(m/chunk_rows) int32, zeroed by the call (stream-ordered memset); one
+ * call at a time per workspace.
+ * The fused kernel needs world <= 8, shard boundaries on chunk boundaries,
+ * k % 8 == 0, 16-B aligned A, peers, B and C and the hgemm() tensor-core
+ * preconditions; otherwise (or for a quick return) the peers' rows are copied
+ * on `stream` first (cudaMemcpy2DAsync) and hgemm() runs unfused.  Asynchronous
+ * like hgemm().
+ * Errors (synchronous, nothing enqueued): HGEMM_ERR_INVALID_VALUE for the
+ * hgemm() argument errors, world < 1, rank outside [0, world), bad
+ * row_splits, chunk_rows < 1, workspace too small, NULL workspace / A / a
+ * needed peer pointer; HGEMM_ERR_ARCH; HGEMM_ERR_CUDA. */
+hgemm_status_t hgemm_allgather_a(int64_t m, int64_t n, int64_t k, float alpha,
+                                 void *A, int64_t lda, const void *const *A_peers,
+                                 const int64_t *row_splits, int32_t world, int32_t rank,
+                                 const void *B, int64_t ldb, float beta, void *C, int64_t ldc,
+                                 char transB, hgemm_dtype_t out_dtype,
+                                 int32_t *workspace, int64_t workspace_ints, int64_t chunk_rows,
+                                 cudaStream_t stream);
+
+/* The chunk order of hgemm_allgather_a (the unfused copies follow it, the
+ * fused kernel's work index and tile raster follow the same owner rotation),
+ * as data (host only, no GPU needed).
+ * Writes up to max_ops records of 4 int64 {chunk, src_rank, row0, row1} to
+ * `ops` in issue order and the total count to *num_ops.  The records of one
+ * chunk are consecutive.  A record
+ * with src_rank == rank covers rows already local (no copy).  Every row of
+ * [0, m) appears in exactly one record, with its owner as src_rank.
+ * ops may be NULL (count only).  Errors: HGEMM_ERR_INVALID_VALUE as above. */
+hgemm_status_t hgemm_allgather_plan(int64_t m, const int64_t *row_splits, int32_t world, int32_t rank,
+                                    int64_t chunk_rows, int64_t *ops, int64_t max_ops, int64_t *num_ops);
+
+/* CUDA IPC of device buffers (cudaIpcGetMemHandle / cudaIpcOpenMemHandle),
+ * for interior pointers of an allocation: the handle carries the offset of
+ * `dptr` from its allocation base (cuMemGetAddressRange).  The handle is
+ * plain bytes: exchange it between processes by any means (the Python
+ * layer uses torch.distributed.all_gather_object).  hgemm_ipc_open maps a
+ * peer's buffer into this process (peer access enabled lazily) and returns
+ * the pointer matching the peer's dptr; hgemm_ipc_close unmaps it.
+ * Errors: HGEMM_ERR_INVALID_VALUE (NULL arguments, unknown pointer),
+ * HGEMM_ERR_CUDA. */
+typedef struct {
+    unsigned char handle[64];  /* cudaIpcMemHandle_t */
+    int64_t offset;            /* dptr - allocation base, bytes */
+} hgemm_ipc_handle_t;
+hgemm_status_t hgemm_ipc_get_handle(const void *dptr, hgemm_ipc_handle_t *out);
+hgemm_status_t hgemm_ipc_open(const hgemm_ipc_handle_t *h, void **dptr);
+hgemm_status_t hgemm_ipc_close(void *dptr);
+
 #ifdef __cplusplus
 }
 #endif

@@ -32,6 +32,11 @@ class _Config(ctypes.Structure):
                 ("stream_k", ctypes.c_int32)]
 
 
+class IpcHandle(ctypes.Structure):
+    """hgemm_ipc_handle_t: cudaIpcMemHandle_t bytes + offset from the allocation base."""
+    _fields_ = [("handle", ctypes.c_ubyte * 64), ("offset", ctypes.c_int64)]
+
+
 def lib_path() -> str:
     return os.environ.get("HGEMM_LIB", os.path.join(_PKG, "libhgemm.so"))
 
@@ -73,6 +78,19 @@ def load_library():
     lib.hgemm_set_probe.restype = ctypes.c_int
     lib.hgemm_launch_count.argtypes = []
     lib.hgemm_launch_count.restype = ctypes.c_int64
+    i32, pi64 = ctypes.c_int32, ctypes.POINTER(ctypes.c_int64)
+    lib.hgemm_allgather_a.argtypes = [i64, i64, i64, f32, vp, i64, ctypes.POINTER(vp), pi64, i32, i32,
+                                      vp, i64, f32, vp, i64, ctypes.c_char, ctypes.c_int,
+                                      vp, i64, i64, vp]
+    lib.hgemm_allgather_a.restype = ctypes.c_int
+    lib.hgemm_allgather_plan.argtypes = [i64, pi64, i32, i32, i64, pi64, i64, pi64]
+    lib.hgemm_allgather_plan.restype = ctypes.c_int
+    lib.hgemm_ipc_get_handle.argtypes = [vp, ctypes.POINTER(IpcHandle)]
+    lib.hgemm_ipc_get_handle.restype = ctypes.c_int
+    lib.hgemm_ipc_open.argtypes = [ctypes.POINTER(IpcHandle), ctypes.POINTER(vp)]
+    lib.hgemm_ipc_open.restype = ctypes.c_int
+    lib.hgemm_ipc_close.argtypes = [vp]
+    lib.hgemm_ipc_close.restype = ctypes.c_int
     _lib = lib
     return lib
 
@@ -219,3 +237,61 @@ def hgemm_torch(A, B, C=None, *, alpha=1.0, beta=0.0, out_dtype=None, stream=Non
     out = HGEMM_OUT_F32 if C.dtype == torch.float32 else HGEMM_OUT_F16
     hgemm(N, M, K, alpha, Bt, lda, At, ldb, beta, C, ldc, tA, tB, out, stream)
     return C
+
+
+def _i64_array(vals):
+    return (ctypes.c_int64 * len(vals))(*[int(v) for v in vals])
+
+
+def allgather_plan(m, row_splits, rank, chunk_rows):
+    """Chunk order of hgemm_allgather_a (host only): list of (chunk, src_rank, row0, row1)."""
+    lib = load_library()
+    world = len(row_splits) - 1
+    rs = _i64_array(row_splits)
+    cnt = ctypes.c_int64(0)
+    _check(lib.hgemm_allgather_plan(int(m), rs, int(world), int(rank), int(chunk_rows), None, 0, ctypes.byref(cnt)))
+    ops = (ctypes.c_int64 * (4 * max(cnt.value, 1)))()
+    _check(lib.hgemm_allgather_plan(int(m), rs, int(world), int(rank), int(chunk_rows), ops, cnt.value,
+                                    ctypes.byref(cnt)))
+    return [tuple(ops[4 * i:4 * i + 4]) for i in range(cnt.value)]
+
+
+def hgemm_allgather_a(m, n, k, alpha, A, lda, A_peers, row_splits, rank, B, ldb, beta, C, ldc,
+                      transB="N", out_dtype=HGEMM_OUT_F16, *, workspace, chunk_rows, stream=None):
+    """All-gather of op(A) rows fused with the GEMM in one kernel (include/hgemm.h hgemm_allgather_a).
+
+    A: this rank's full-size gather buffer (transA = 'T' layout); A_peers: the
+    other ranks' gather buffers as device pointers/tensors (entry `rank` ignored);
+    workspace: int32 CUDA tensor of >= 1 + ceil(m/chunk_rows) entries."""
+    lib = load_library()
+    world = len(row_splits) - 1
+    if len(A_peers) != world:
+        raise HgemmError("A_peers needs one entry per rank")
+    peers = (ctypes.c_void_p * world)(*[_ptr(x) or None for x in A_peers])
+    nws = int(workspace.numel()) if hasattr(workspace, "numel") else 0
+    code = lib.hgemm_allgather_a(int(m), int(n), int(k), float(alpha), _ptr(A), int(lda), peers,
+                                 _i64_array(row_splits), int(world), int(rank), _ptr(B), int(ldb), float(beta),
+                                 _ptr(C), int(ldc), transB.encode()[:1], _out_code(out_dtype), _ptr(workspace), nws,
+                                 int(chunk_rows), _stream(stream))
+    _check(code)
+
+
+def ipc_get_handle(buf) -> bytes:
+    """72 bytes (hgemm_ipc_handle_t) naming the device buffer `buf` for other processes."""
+    h = IpcHandle()
+    _check(load_library().hgemm_ipc_get_handle(_ptr(buf), ctypes.byref(h)))
+    return bytes(ctypes.string_at(ctypes.addressof(h), ctypes.sizeof(h)))
+
+
+def ipc_open(handle: bytes) -> int:
+    """Map a peer's buffer (from ipc_get_handle) into this process; returns its device pointer."""
+    if len(handle) != ctypes.sizeof(IpcHandle):
+        raise HgemmError("bad IPC handle size")
+    h = IpcHandle.from_buffer_copy(handle)
+    out = ctypes.c_void_p()
+    _check(load_library().hgemm_ipc_open(ctypes.byref(h), ctypes.byref(out)))
+    return int(out.value)
+
+
+def ipc_close(ptr: int):
+    _check(load_library().hgemm_ipc_close(ctypes.c_void_p(int(ptr))))

@@ -206,12 +206,13 @@ bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags)
 }
 
 // ----------------------------------------------------------------- TC launch
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC>
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC, bool AG = false>
 hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &td, const TcParams &p0,
                          int dev, const DeviceInfo &di, int max_ctas, int sk_mode, bool *sk_used,
                          cudaStream_t stream) {
   using S = TcShape<BN, CG, OUT_F32>;
-  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC>;
+  constexpr int THREADS = S::THREADS + (AG ? 32 : 0);  // + the all-gather copy warp
+  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC, AG>;
   static int attr_done[kMaxDevices] = {};
   static int max_clusters[kMaxDevices] = {};
   if (!attr_done[dev]) {
@@ -220,7 +221,7 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
     if (CG == 2) {
       cudaLaunchConfig_t qc = {};
       qc.gridDim = dim3(CG * MC * (di.num_sms / (CG * MC)));
-      qc.blockDim = dim3(S::THREADS);
+      qc.blockDim = dim3(THREADS);
       qc.dynamicSmemBytes = S::SMEM_BYTES;
       cudaLaunchAttribute qa[1];
       qa[0].id = cudaLaunchAttributeClusterDimension;
@@ -247,7 +248,7 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   p.sk_ws = nullptr;
   p.sk_flags = nullptr;
   *sk_used = false;
-  if (MC == 1) {
+  if (MC == 1 && !AG) {
     const int dp = sk_plan(tiles, units, p.num_k_blocks, sk_mode);
     float *ws = nullptr;
     int *flags = nullptr;
@@ -263,7 +264,7 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(clusters * CG * MC);
-  cfg.blockDim = dim3(S::THREADS);
+  cfg.blockDim = dim3(THREADS);
   cfg.dynamicSmemBytes = S::SMEM_BYTES;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
@@ -295,6 +296,17 @@ hgemm_status_t dispatch_tc_layout(bool a_mn, bool b_mn, bool f32, const CUtensor
   HG_CASE(true, true, true)
 #undef HG_CASE
   return HGEMM_ERR_INVALID_VALUE;
+}
+
+// fused all-gather kernels: CTA pairs, op(A) K-major (transA = 'T')
+template <int BN>
+hgemm_status_t dispatch_tc_ag(bool a_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
+                              const CUtensorMap &td, const TcParams &p, int dev, const DeviceInfo &di, int max_ctas,
+                              bool *sk_used, cudaStream_t s) {
+  if (!a_mn && !f32) return launch_tc<BN, 2, false, false, false, 1, true>(ta, tb, td, p, dev, di, max_ctas, 1, sk_used, s);
+  if (!a_mn && f32) return launch_tc<BN, 2, false, false, true, 1, true>(ta, tb, td, p, dev, di, max_ctas, 1, sk_used, s);
+  if (a_mn && !f32) return launch_tc<BN, 2, true, false, false, 1, true>(ta, tb, td, p, dev, di, max_ctas, 1, sk_used, s);
+  return launch_tc<BN, 2, true, false, true, 1, true>(ta, tb, td, p, dev, di, max_ctas, 1, sk_used, s);
 }
 
 // ----------------------------------------------------------------- split-K launch
@@ -509,9 +521,24 @@ hgemm_status_t hgemm_set_probe(unsigned long long *device_buf) {
   return HGEMM_SUCCESS;
 }
 
-hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A, int64_t lda, const void *B,
-                     int64_t ldb, float beta, void *C, int64_t ldc, char transA, char transB,
-                     hgemm_dtype_t out_dtype, cudaStream_t stream) {
+}  // extern "C"
+
+namespace {
+
+// Fused all-gather of op(A) (hgemm_allgather_a): the kernel waits per chunk of
+// op(A) rows for the copy stream's flag; raster groups along N, one group per
+// chunk, starting with the group of this rank's first local chunk.
+struct AgSpec {
+  int *ctr;                 // [0] work index, [1 + c] finished copy units of chunk c (zeroed)
+  const void *const *peers;
+  const int64_t *rs;
+  int world, rank;
+  int64_t chunk_rows, unit_rows, units;
+};
+
+hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const void *A, int64_t lda,
+                          const void *B, int64_t ldb, float beta, void *C, int64_t ldc, char transA, char transB,
+                          hgemm_dtype_t out_dtype, cudaStream_t stream, const AgSpec *ag) {
   // ---------------------------------------------------------- validation (no side effects)
   if (m < 0 || n < 0 || k < 0) return HGEMM_ERR_INVALID_VALUE;
   if (!(is_t(transA) || is_n(transA)) || !(is_t(transB) || is_n(transB))) return HGEMM_ERR_INVALID_VALUE;
@@ -560,7 +587,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   const bool tc_ok = aligned16(A) && aligned16(B) && aligned16(C) && (lda % 8 == 0) && (ldb % 8 == 0) &&
                      ((ldc * out_size) % 16 == 0) && m < (1ll << 31) && n < (1ll << 31) && k < (1ll << 31) &&
                      lda < (1ll << 36) && ldb < (1ll << 36) && ldc < (1ll << 36) && encode_fn() != nullptr;
-  const bool want_simt = (cfg.kernel == HGEMM_KERNEL_SIMT);
+  const bool want_simt = !ag && (cfg.kernel == HGEMM_KERNEL_SIMT);
   if (!tc_ok || want_simt) {
     dim3 grid(static_cast<unsigned>(cdiv(m, 64)), static_cast<unsigned>(cdiv(n, 64)));
     if (grid.y > 65535u) return HGEMM_ERR_INVALID_VALUE;
@@ -581,7 +608,7 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   const bool b_mn = !tA;  // Bk = op(A):   'N' -> rows of Bk contiguous along N
 
   // ---------------------------------------------------------- HBM streaming (skinny, TN)
-  if (!a_mn && !b_mn && M <= 256 &&
+  if (!ag && !a_mn && !b_mn && M <= 256 &&
       ((cfg.kernel == HGEMM_KERNEL_STREAM) ||
        (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream(M, N, k, di.num_sms)))) {
     const int mt = M <= 128 ? 1 : 2;
@@ -630,7 +657,9 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   {
     int sk_bn = 0, sk_spl = 0;
     bool use_sk = false;
-    if (cfg.kernel == HGEMM_KERNEL_SPLITK) {
+    if (ag) {
+      // the fused all-gather runs the persistent tile kernel only
+    } else if (cfg.kernel == HGEMM_KERNEL_SPLITK) {
       use_sk = true;
       sk_bn = cfg.block_n ? cfg.block_n : (N <= 64 ? 64 : 128);
       sk_spl = cfg.splits ? cfg.splits : 4;
@@ -670,16 +699,19 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   }
 
   int cg = 2, bn = 512;
-  const int forced_cg = cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
-  if (forced_cg && cfg.block_n) { cg = forced_cg; bn = cfg.block_n; }
-  else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, cfg.stream_k, cg, bn);
+  // the fused all-gather kernels exist for CTA pairs only
+  const int forced_cg = ag ? 2 : cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
+  // stream-K is off under the fused all-gather (its work items do not follow the chunk order)
+  const int skm = ag ? 1 : cfg.stream_k;
+  if (forced_cg && cfg.block_n && !(ag && cfg.block_n == 128)) { cg = forced_cg; bn = cfg.block_n; }
+  else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, skm, cg, bn);
   const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
   // MC = 2: two CTA pairs per cluster share (multicast) the Bk half-boxes
   // (measured slower everywhere: a 4-CTA cluster strands SMs of the GPCs and couples
   // the two pairs' pipelines; built only with -DHGEMM_ENABLE_MC)
   int mc = 1;
 #ifdef HGEMM_ENABLE_MC
-  if (cg == 2) {
+  if (cg == 2 && !ag) {
     if (const char *e = std::getenv("HGEMM_MC")) mc = std::atoi(e) == 2 ? 2 : 1;  // experiments
   }
 #endif
@@ -714,6 +746,27 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     const char *e = std::getenv("HGEMM_L2_HINT");
     p.l2_hint = e ? std::atoi(e) : 0;
   }
+  if (ag) {
+    p.ag_ctr = ag->ctr;
+    for (int q = 0; q < ag->world; ++q) p.ag_peer[q] = ag->peers[q];
+    for (int q = 0; q <= ag->world; ++q) p.ag_rs[q] = ag->rs[q];
+    p.ag_A = const_cast<void *>(A);
+    p.ag_lda = lda;
+    p.ag_world = ag->world;
+    p.ag_rank = ag->rank;
+    p.ag_chunk_rows = static_cast<int32_t>(ag->chunk_rows);
+    p.ag_unit_rows = static_cast<int32_t>(ag->unit_rows);
+    p.ag_units = static_cast<int32_t>(ag->units);
+    // one raster group per chunk (bn-aligned chunks tiling N exactly), starting with
+    // this rank's first chunk, so the tiles run in the order the copies complete
+    if (ag->chunk_rows % bn == 0) {
+      const int gn = static_cast<int>(ag->chunk_rows / bn);
+      if (gn <= p.num_n_tiles && p.num_n_tiles % gn == 0) {
+        p.group_m = -gn;
+        p.n_rot = static_cast<int32_t>((ag->rs[ag->rank] / ag->chunk_rows) % (p.num_n_tiles / gn));
+      }
+    }
+  }
   p.probe = g_probe.load(std::memory_order_relaxed);
   p.alpha = alpha;
   p.beta = beta;
@@ -722,7 +775,6 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
 
   hgemm_status_t st;
   bool sk_used = false;
-  const int skm = cfg.stream_k;
 #ifdef HGEMM_ENABLE_MC
   if (cg == 2 && bn == 512 && mc == 2)
     st = dispatch_tc_layout<512, 2, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
@@ -730,7 +782,10 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     st = dispatch_tc_layout<256, 2, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
   else
 #endif
-  if (cg == 2 && bn == 512)
+  if (ag)
+    st = bn == 512 ? dispatch_tc_ag<512>(a_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, &sk_used, stream)
+                   : dispatch_tc_ag<256>(a_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, &sk_used, stream);
+  else if (cg == 2 && bn == 512)
     st = dispatch_tc_layout<512, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
   else if (cg == 2)
     st = dispatch_tc_layout<256, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
@@ -743,6 +798,16 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
     g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0, sk_used ? 2 : 1};
   }
   return st;
+}
+
+}  // namespace
+
+extern "C" {
+
+hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A, int64_t lda, const void *B,
+                     int64_t ldb, float beta, void *C, int64_t ldc, char transA, char transB,
+                     hgemm_dtype_t out_dtype, cudaStream_t stream) {
+  return hgemm_core(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA, transB, out_dtype, stream, nullptr);
 }
 
 }  // extern "C"
@@ -885,6 +950,218 @@ hgemm_status_t hgemm_host(int64_t m, int64_t n, int64_t k, float alpha, const vo
   if (cudaStreamWaitEvent(stream, P.ev_comp[HostPipe::kEv - 1], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
   if (cudaStreamSynchronize(P.s_out) != cudaSuccess) return HGEMM_ERR_CUDA;
   return HGEMM_SUCCESS;
+}
+
+}  // extern "C"
+
+// ============================================================================
+// Sharded path: all-gather of op(A) fused with the GEMM (include/hgemm.h;
+// BASELINE.json north_star (3), DESIGN.md "Fused
+// all-gather").  The copy engines pull the peers' rows of op(A) over NVLink
+// into the local gather buffer chunk by chunk and raise one flag per chunk;
+// the persistent GEMM kernel (already running) waits per tile for the chunks
+// it reads.  No SM is spent on the transfer and no NCCL kernel has to share
+// the SMs with the persistent GEMM.
+namespace {
+
+bool plan_args_ok(int64_t m, const int64_t *row_splits, int32_t world, int32_t rank, int64_t chunk_rows) {
+  if (m < 0 || world < 1 || rank < 0 || rank >= world || chunk_rows < 1 || !row_splits) return false;
+  if (row_splits[0] != 0 || row_splits[world] != m) return false;
+  for (int q = 0; q < world; ++q)
+    if (row_splits[q + 1] < row_splits[q]) return false;
+  return true;
+}
+
+int owner_of(int64_t row, const int64_t *row_splits, int32_t world) {
+  int q = 0;
+  while (q + 1 < world && row >= row_splits[q + 1]) ++q;
+  return q;
+}
+
+// Issue order: chunks grouped by the owner of their first row, owners in the
+// order rank, rank+1, ... (mod world) so the local chunks come first and the
+// ranks pull from different peers at any moment; within a chunk one record per
+// owner segment.
+template <typename F>
+void plan_walk(int64_t m, const int64_t *row_splits, int32_t world, int32_t rank, int64_t chunk_rows, F &&emit) {
+  const int64_t nchunks = (m + chunk_rows - 1) / chunk_rows;
+  for (int d = 0; d < world; ++d) {
+    const int q = (rank + d) % world;
+    for (int64_t c = 0; c < nchunks; ++c) {
+      const int64_t c0 = c * chunk_rows, c1 = std::min(m, c0 + chunk_rows);
+      if (owner_of(c0, row_splits, world) != q) continue;
+      int64_t r = c0;
+      while (r < c1) {
+        const int o = owner_of(r, row_splits, world);
+        const int64_t e = std::min(c1, row_splits[o + 1]);
+        emit(c, o, r, e);
+        r = e;
+      }
+    }
+  }
+}
+
+using MemGetAddressRangeFn = CUresult (*)(CUdeviceptr *, size_t *, CUdeviceptr);
+
+template <typename Fn>
+Fn driver_fn(const char *name) {
+  void *p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPointByVersion(name, &p, 12000, cudaEnableDefault, &q) != cudaSuccess ||
+      q != cudaDriverEntryPointSuccess)
+    return nullptr;
+  return reinterpret_cast<Fn>(p);
+}
+
+struct IpcMapping {
+  void *user;
+  void *base;
+};
+std::mutex g_ipc_mu;
+IpcMapping g_ipc[256];
+int g_ipc_n = 0;
+
+}  // namespace
+
+extern "C" {
+
+hgemm_status_t hgemm_allgather_plan(int64_t m, const int64_t *row_splits, int32_t world, int32_t rank,
+                                    int64_t chunk_rows, int64_t *ops, int64_t max_ops, int64_t *num_ops) {
+  if (!num_ops || !plan_args_ok(m, row_splits, world, rank, chunk_rows)) return HGEMM_ERR_INVALID_VALUE;
+  int64_t cnt = 0;
+  plan_walk(m, row_splits, world, rank, chunk_rows, [&](int64_t c, int o, int64_t r0, int64_t r1) {
+    if (ops && cnt < max_ops) {
+      ops[4 * cnt + 0] = c;
+      ops[4 * cnt + 1] = o;
+      ops[4 * cnt + 2] = r0;
+      ops[4 * cnt + 3] = r1;
+    }
+    ++cnt;
+  });
+  *num_ops = cnt;
+  return HGEMM_SUCCESS;
+}
+
+hgemm_status_t hgemm_allgather_a(int64_t m, int64_t n, int64_t k, float alpha, void *A, int64_t lda,
+                                 const void *const *A_peers, const int64_t *row_splits, int32_t world, int32_t rank,
+                                 const void *B, int64_t ldb, float beta, void *C, int64_t ldc, char transB,
+                                 hgemm_dtype_t out_dtype, int32_t *workspace, int64_t workspace_ints,
+                                 int64_t chunk_rows, cudaStream_t stream) {
+  // ---------------------------------------------------------- validation (no side effects)
+  if (m < 0 || n < 0 || k < 0) return HGEMM_ERR_INVALID_VALUE;
+  if (!(is_t(transB) || is_n(transB))) return HGEMM_ERR_INVALID_VALUE;
+  if (out_dtype != HGEMM_OUT_F16 && out_dtype != HGEMM_OUT_F32) return HGEMM_ERR_INVALID_VALUE;
+  if (lda < std::max<int64_t>(1, k)) return HGEMM_ERR_INVALID_VALUE;
+  if (ldb < std::max<int64_t>(1, is_t(transB) ? n : k)) return HGEMM_ERR_INVALID_VALUE;
+  if (ldc < std::max<int64_t>(1, m)) return HGEMM_ERR_INVALID_VALUE;
+  if (!plan_args_ok(m, row_splits, world, rank, chunk_rows)) return HGEMM_ERR_INVALID_VALUE;
+  const int64_t nchunks = (m + chunk_rows - 1) / chunk_rows;
+  if (!workspace || workspace_ints < 1 + nchunks) return HGEMM_ERR_INVALID_VALUE;
+  if (m > 0 && k > 0 && !A) return HGEMM_ERR_INVALID_VALUE;
+  for (int q = 0; q < world; ++q)
+    if (q != rank && row_splits[q + 1] > row_splits[q] && k > 0 && (!A_peers || !A_peers[q]))
+      return HGEMM_ERR_INVALID_VALUE;
+  if (m > 0 && n > 0 && !C) return HGEMM_ERR_INVALID_VALUE;
+  if (m > 0 && n > 0 && k > 0 && alpha != 0.0f && !B) return HGEMM_ERR_INVALID_VALUE;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return HGEMM_ERR_CUDA;
+  DeviceInfo di;
+  if (!device_info(dev, di)) return HGEMM_ERR_CUDA;
+  if (!di.ok) return HGEMM_ERR_ARCH;
+
+  // ---------------------------------------------------------- fused: one kernel gathers and multiplies
+  const bool f32 = (out_dtype == HGEMM_OUT_F32);
+  const int out_size = f32 ? 4 : 2;
+  bool aligned_shards = world <= 8;
+  for (int q = 1; q < world && aligned_shards; ++q)
+    if (row_splits[q] % chunk_rows != 0 && row_splits[q] != m) aligned_shards = false;
+  bool peers_aligned = true;
+  for (int q = 0; q < world; ++q)
+    if (q != rank && A_peers && !aligned16(A_peers[q])) peers_aligned = false;
+  const bool fused = aligned_shards && peers_aligned && m > 0 && n > 0 && k > 0 && alpha != 0.0f && (k % 8 == 0) &&
+                     aligned16(A) && aligned16(B) && aligned16(C) && (lda % 8 == 0) && (ldb % 8 == 0) &&
+                     ((ldc * out_size) % 16 == 0) && m < (1ll << 31) && n < (1ll << 31) && k < (1ll << 31) &&
+                     lda < (1ll << 36) && ldb < (1ll << 36) && ldc < (1ll << 36) && chunk_rows < (1ll << 30) &&
+                     encode_fn() != nullptr;
+  if (fused) {
+    // copy unit: ~64 KB of rows, a power of two dividing chunk_rows (never straddles a chunk)
+    const int64_t target = std::max<int64_t>(1, 65536 / (k * 2));
+    int64_t u = 1;
+    while (u * 2 <= target && chunk_rows % (u * 2) == 0) u *= 2;
+    int64_t units = 0;
+    for (int q = 0; q < world; ++q)
+      if (q != rank) units += (row_splits[q + 1] - row_splits[q] + u - 1) / u;
+    if (units < (1ll << 31)) {
+      if (cudaMemsetAsync(workspace, 0, static_cast<size_t>(1 + nchunks) * 4, stream) != cudaSuccess)
+        return HGEMM_ERR_CUDA;
+      const AgSpec ag = {workspace, A_peers, row_splits, world, rank, chunk_rows, u, units};
+      return hgemm_core(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, 'T', transB, out_dtype, stream, &ag);
+    }
+  }
+
+  // ---------------------------------------------------------- unfused: copies, then hgemm()
+  const size_t pitch = static_cast<size_t>(lda) * 2;
+  hgemm_status_t st = HGEMM_SUCCESS;
+  if (k > 0) {
+    plan_walk(m, row_splits, world, rank, chunk_rows, [&](int64_t, int o, int64_t r0, int64_t r1) {
+      if (st != HGEMM_SUCCESS || o == rank) return;
+      const char *src = static_cast<const char *>(A_peers[o]) + static_cast<size_t>(r0) * pitch;
+      char *dst = static_cast<char *>(A) + static_cast<size_t>(r0) * pitch;
+      if (cudaMemcpy2DAsync(dst, pitch, src, pitch, static_cast<size_t>(k) * 2, static_cast<size_t>(r1 - r0),
+                            cudaMemcpyDeviceToDevice, stream) != cudaSuccess)
+        st = HGEMM_ERR_CUDA;
+    });
+  }
+  if (st != HGEMM_SUCCESS) return st;
+  return hgemm_core(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, 'T', transB, out_dtype, stream, nullptr);
+}
+
+hgemm_status_t hgemm_ipc_get_handle(const void *dptr, hgemm_ipc_handle_t *out) {
+  if (!dptr || !out) return HGEMM_ERR_INVALID_VALUE;
+  static MemGetAddressRangeFn range = driver_fn<MemGetAddressRangeFn>("cuMemGetAddressRange");
+  if (!range) return HGEMM_ERR_CUDA;
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (range(&base, &size, reinterpret_cast<CUdeviceptr>(dptr)) != CUDA_SUCCESS) return HGEMM_ERR_INVALID_VALUE;
+  cudaIpcMemHandle_t h;
+  if (cudaIpcGetMemHandle(&h, reinterpret_cast<void *>(base)) != cudaSuccess) return HGEMM_ERR_CUDA;
+  static_assert(sizeof(h) == sizeof(out->handle), "cudaIpcMemHandle_t size");
+  std::memcpy(out->handle, &h, sizeof(h));
+  out->offset = static_cast<int64_t>(reinterpret_cast<CUdeviceptr>(dptr) - base);
+  return HGEMM_SUCCESS;
+}
+
+hgemm_status_t hgemm_ipc_open(const hgemm_ipc_handle_t *h, void **dptr) {
+  if (!h || !dptr || h->offset < 0) return HGEMM_ERR_INVALID_VALUE;
+  cudaIpcMemHandle_t ch;
+  std::memcpy(&ch, h->handle, sizeof(ch));
+  void *base = nullptr;
+  if (cudaIpcOpenMemHandle(&base, ch, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) return HGEMM_ERR_CUDA;
+  void *user = static_cast<char *>(base) + h->offset;
+  std::lock_guard<std::mutex> lk(g_ipc_mu);
+  if (g_ipc_n == static_cast<int>(sizeof(g_ipc) / sizeof(g_ipc[0]))) {
+    cudaIpcCloseMemHandle(base);
+    return HGEMM_ERR_CUDA;
+  }
+  g_ipc[g_ipc_n++] = {user, base};
+  *dptr = user;
+  return HGEMM_SUCCESS;
+}
+
+hgemm_status_t hgemm_ipc_close(void *dptr) {
+  if (!dptr) return HGEMM_ERR_INVALID_VALUE;
+  void *base = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(g_ipc_mu);
+    for (int i = 0; i < g_ipc_n; ++i)
+      if (g_ipc[i].user == dptr) {
+        base = g_ipc[i].base;
+        g_ipc[i] = g_ipc[--g_ipc_n];
+        break;
+      }
+  }
+  if (!base) return HGEMM_ERR_INVALID_VALUE;
+  return cudaIpcCloseMemHandle(base) == cudaSuccess ? HGEMM_SUCCESS : HGEMM_ERR_CUDA;
 }
 
 }  // extern "C"

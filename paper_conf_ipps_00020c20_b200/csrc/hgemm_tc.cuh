@@ -61,6 +61,23 @@ struct TcParams {
   int64_t sk_u0, sk_units;
   float *sk_ws;                      // one 128 x BN FP32 partial-accumulator slot per CTA
   int *sk_flags;                     // one flag per CTA: 1 = slot published; consumers reset it to 0
+  // Fused all-gather of op(A) (hgemm_allgather_a, kernels with AG = true; DESIGN.md
+  // "Fused all-gather").  Bk = op(A) is this rank's gather buffer ag_A (row r at
+  // ag_A + r*ag_lda); rank q owns rows [ag_rs[q], ag_rs[q+1]) (chunk-aligned).  The
+  // copy warp of every CTA pulls the peers' rows from ag_peer[q] in units of
+  // ag_unit_rows rows (a unit never straddles a chunk), taking units from the
+  // shared work index ag_ctr[0] in the order owners rank+1, rank+2, ...; after a
+  // unit it adds 1 to ag_ctr[1 + chunk].  A tile's TMA loads of chunk c wait for
+  // ag_ctr[1 + c] to reach the chunk's unit count.  ag_ctr is zeroed per call.
+  int *ag_ctr;
+  const void *ag_peer[8];
+  int64_t ag_rs[9];
+  void *ag_A;
+  int64_t ag_lda;
+  int32_t ag_world, ag_rank;
+  int32_t ag_chunk_rows, ag_unit_rows;
+  int32_t ag_units;                  // copy units in total (all peers)
+  int32_t n_rot;                     // raster groups along N start at group n_rot (group_m < 0 only)
 };
 
 // One unit of work of a cluster: k-blocks [kb0, kb1) of cluster tile `tile`.
@@ -135,10 +152,12 @@ __device__ __forceinline__ void tile_coords(int t, const TcParams &p, int &tm, i
     // grouped along N: -group_m n-tiles per group, n fastest
     const int gn = -p.group_m;
     const int per_group = gn * p.num_m_tiles;
-    const int g = t / per_group;
+    int g = t / per_group;
+    const int r = t - g * per_group;
+    // rotation (all groups full-size, checked by the host): start with group n_rot
+    if (p.n_rot != 0) g = (g + p.n_rot) % (p.num_n_tiles / gn);
     const int first_n = g * gn;
     const int gsz = min(p.num_n_tiles - first_n, gn);
-    const int r = t - g * per_group;
     tn = first_n + r % gsz;
     tm = r / gsz;
     return;
@@ -282,8 +301,59 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
 // from (16 + 2*16) KB to (16 + 16) KB per k-block for BN = 512 (DESIGN.md
 // "Multicast").  A stage may be overwritten only after both pairs' MMAs have
 // read it: empty[] counts MC arrivals, multicast by each pair's MMA leader.
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC = 1>
-__global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
+// Copy warp of the fused all-gather (AG = true; warp 2 + EPI_WARPS): pulls copy
+// units of op(A) rows from the peers' gather buffers (over NVLink: plain 16-B
+// loads from P2P-mapped memory) into the local one, 8 loads in flight per lane,
+// and publishes each finished unit in its chunk's counter.  Units are taken from
+// a shared work index, so any subset of resident CTAs completes all of them.
+__device__ __forceinline__ void ag_copy_warp(const TcParams &p, uint32_t lane) {
+  const int64_t vpr = static_cast<int64_t>(p.K) / 8;  // 16-B vectors per row (K % 8 == 0)
+  const int64_t ld_v = p.ag_lda / 8;
+  for (;;) {
+    int u = 0;
+    if (lane == 0) u = atomicAdd(p.ag_ctr, 1);
+    u = __shfl_sync(0xffffffffu, u, 0);
+    if (u >= p.ag_units) break;
+    // owner of unit u: peers in the order rank+1, rank+2, ...
+    int q = p.ag_rank;
+    int64_t j = u;
+    for (int d = 1; d < p.ag_world; ++d) {
+      q = (p.ag_rank + d) % p.ag_world;
+      const int64_t nq = (p.ag_rs[q + 1] - p.ag_rs[q] + p.ag_unit_rows - 1) / p.ag_unit_rows;
+      if (j < nq) break;
+      j -= nq;
+    }
+    const int64_t r0 = p.ag_rs[q] + j * p.ag_unit_rows;
+    const int64_t r1 = min(p.ag_rs[q + 1], r0 + p.ag_unit_rows);
+    const uint4 *src = static_cast<const uint4 *>(p.ag_peer[q]);
+    uint4 *dst = static_cast<uint4 *>(p.ag_A);
+    const int64_t total = (r1 - r0) * vpr;
+    constexpr int UNR = 8;
+    for (int64_t base = 0; base < total; base += 32 * UNR) {
+      uint4 v[UNR];
+      int64_t off[UNR];
+#pragma unroll
+      for (int i = 0; i < UNR; ++i) {
+        const int64_t e = base + lane + 32 * i;
+        const int64_t row = r0 + e / vpr;
+        off[i] = e < total ? row * ld_v + (e - (row - r0) * vpr) : -1;
+        if (off[i] >= 0) v[i] = src[off[i]];
+      }
+#pragma unroll
+      for (int i = 0; i < UNR; ++i)
+        if (off[i] >= 0) dst[off[i]] = v[i];
+    }
+    fence_proxy_async_global();
+    __syncwarp();
+    if (lane == 0) {
+      __threadfence();
+      atomicAdd(p.ag_ctr + 1 + static_cast<int>(r0 / p.ag_chunk_rows), 1);
+    }
+  }
+}
+
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC = 1, bool AG = false>
+__global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 : 0), 1)
     hgemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmD, const TcParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
@@ -381,6 +451,19 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
         tile_coords(wi.tile, p, tm, tn);
         const int a_row = (tm * MC + static_cast<int>(pair)) * BM * CG + static_cast<int>(prank) * BM;
         const int b_row0 = tn * BN + static_cast<int>(prank) * B_ROWS;
+        if constexpr (AG) {
+          // fused all-gather: wait until every chunk of op(A) rows this tile reads
+          // (tn*BN .. +BN) is complete in the local gather buffer
+          const int r0 = tn * BN, r1 = min(p.N, r0 + BN) - 1;
+          for (int c = r0 / p.ag_chunk_rows; c <= r1 / p.ag_chunk_rows; ++c) {
+            const int64_t c0 = static_cast<int64_t>(c) * p.ag_chunk_rows;
+            if (c0 >= p.ag_rs[p.ag_rank] && c0 < p.ag_rs[p.ag_rank + 1]) continue;  // local rows
+            const int rows = static_cast<int>(min(static_cast<int64_t>(p.N), c0 + p.ag_chunk_rows) - c0);
+            const int need = (rows + p.ag_unit_rows - 1) / p.ag_unit_rows;
+            while (ld_acquire_gpu(p.ag_ctr + 1 + c) < need) __nanosleep(128);
+          }
+          fence_proxy_async_global();  // the copy warps' generic stores -> this CTA's TMA (async proxy) reads
+        }
         for (int kb = wi.kb0; kb < wi.kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1u);
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
@@ -556,6 +639,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS, 1)
 #endif
       }
     }
+  } else if (AG && warp == 2u + S::EPI_WARPS) {
+    // ------------------------------------------------------------ all-gather copy warp
+    if constexpr (AG) ag_copy_warp(p, lane);
   } else {
     // ------------------------------------------------------------ epilogue warps
     const uint32_t quad = warp & 3u;                 // TMEM lane quadrant this warp may access

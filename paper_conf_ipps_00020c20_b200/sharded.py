@@ -148,3 +148,84 @@ def _offset(t, off):
     if isinstance(t, int):
         return t + off
     return _Offset(t, off)
+
+
+def default_chunk_rows(m: int, world: int, bn: int = 512) -> int:
+    """Chunk of op(A) rows per copy-engine transfer / GEMM flag: a multiple of the
+    512-wide tile (one raster group of tiles per chunk), about half a shard."""
+    half_shard = m // max(1, 2 * world)
+    return max(bn, half_shard - half_shard % bn)
+
+
+class FusedAllGatherA:
+    """A replicated by an all-gather fused with the GEMM (hgemm_allgather_a, NEXT-2).
+
+    Rank q owns rows [row_splits[q], row_splits[q+1]) of op(A) (transA = 'T',
+    the paper's layout: A stored k x m, row i of op(A) = A + i*lda).  Every rank
+    allocates a full-size gather buffer `self.A` (a (m, lda) float16 tensor whose
+    row i is op(A) row i) and writes its own rows there; the buffers are mapped
+    into every peer with CUDA IPC once (handles exchanged over the process
+    group).  Each call is ONE kernel: a copy warp per CTA pulls the peers' rows
+    over NVLink while the persistent GEMM of this rank's C slab consumes each
+    chunk of rows as soon as it is complete, so the exchange overlaps the MMAs
+    tile by tile.  The result is bitwise that of hgemm() on the gathered A.
+
+    The caller synchronises the ranks around a call (a barrier after writing its
+    own rows, and before rewriting them while a peer may still be reading).
+    `ipc` = (get_handle, open, close) and `alloc` are injection points for the
+    CPU (gloo) tests of the exchange logic; the defaults are the C ABI and torch."""
+
+    def __init__(self, m: int, k: int, *, lda: int | None = None, group=None, chunk_rows: int | None = None,
+                 device=None, ipc=None, alloc=None):
+        import torch
+        import torch.distributed as dist
+        self.world, self.rank = _world_rank(group)
+        self.m, self.k = int(m), int(k)
+        self.lda = int(lda) if lda is not None else max(1, self.k + (-self.k) % 8)
+        self.chunk_rows = int(chunk_rows) if chunk_rows else default_chunk_rows(self.m, self.world)
+        # shards on chunk boundaries: every chunk has one owner (the fused kernel's precondition)
+        self.row_splits = [slab_bounds(self.m, self.world, q, align=self.chunk_rows)[0] for q in range(self.world)]
+        self.row_splits.append(self.m)
+        nws = 1 + max(1, -(-self.m // self.chunk_rows))
+        if alloc is None:
+            dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+            self.A = torch.empty((self.m, self.lda), dtype=torch.float16, device=dev)
+            self.workspace = torch.zeros(nws, dtype=torch.int32, device=dev)
+        else:
+            self.A, self.workspace = alloc(self.m, self.lda, nws)
+        if ipc is None:
+            from . import binding
+            ipc = (binding.ipc_get_handle, binding.ipc_open, binding.ipc_close)
+        self._get_handle, self._open, self._close = ipc
+        self.peers = [None] * self.world
+        self._opened = []
+        if self.world > 1:
+            mine = self._get_handle(self.A)
+            allh = [None] * self.world
+            dist.all_gather_object(allh, mine, group=group)
+            for q, h in enumerate(allh):
+                if q != self.rank:
+                    self.peers[q] = self._open(h)
+                    self._opened.append(self.peers[q])
+
+    @property
+    def own_rows(self):
+        return self.row_splits[self.rank], self.row_splits[self.rank + 1]
+
+    def own_view(self):
+        """This rank's rows of op(A) inside the gather buffer, to be written by the caller."""
+        r0, r1 = self.own_rows
+        return self.A[r0:r1, :self.k]
+
+    def __call__(self, n, alpha, B, ldb, beta, C, ldc, transB="N", out_dtype="f16", *, stream=None, gemm=None):
+        """C (m x n slab) = alpha * op(A) * op(B) + beta * C with op(A) gathered on the fly."""
+        if gemm is None:
+            from .binding import hgemm_allgather_a as gemm
+        gemm(self.m, n, self.k, alpha, self.A, self.lda, self.peers, self.row_splits, self.rank, B, ldb, beta, C,
+             ldc, transB, out_dtype, workspace=self.workspace, chunk_rows=self.chunk_rows, stream=stream)
+
+    def close(self):
+        for p in self._opened:
+            self._close(p)
+        self._opened = []
+        self.peers = [None] * self.world
