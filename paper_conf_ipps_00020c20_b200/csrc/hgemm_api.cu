@@ -43,6 +43,11 @@ hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
 hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
 std::atomic<int64_t> g_launches{0};
 std::atomic<unsigned long long *> g_probe{nullptr};
+// programmatic dependent launch of the tensor-core kernels (HGEMM_PDL=0 disables it: experiments)
+const bool g_pdl = [] {
+  const char *e = std::getenv("HGEMM_PDL");
+  return !(e && e[0] == '0');
+}();
 
 bool device_info(int dev, DeviceInfo &out) {
   if (dev < 0 || dev >= kMaxDevices) return false;
@@ -267,13 +272,16 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   cfg.blockDim = dim3(THREADS);
   cfg.dynamicSmemBytes = S::SMEM_BYTES;
   cfg.stream = stream;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = CG * MC;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  // programmatic dependent launch: the prologue overlaps the previous kernel's tail
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = 2;
   if (cudaLaunchKernelEx(&cfg, kern, ta, tb, td, p) != cudaSuccess) return HGEMM_ERR_CUDA;
   g_launches.fetch_add(1, std::memory_order_relaxed);
   return HGEMM_SUCCESS;
@@ -328,13 +336,15 @@ hgemm_status_t launch_splitk(const CUtensorMap &ta, const CUtensorMap &tb, const
   cfg.blockDim = dim3(192);
   cfg.dynamicSmemBytes = SH::SMEM_BYTES;
   cfg.stream = stream;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = SPL;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = 2;
   if (cudaLaunchKernelEx(&cfg, kern, ta, tb, p) != cudaSuccess) return HGEMM_ERR_CUDA;
   g_launches.fetch_add(1, std::memory_order_relaxed);
   return HGEMM_SUCCESS;
@@ -403,8 +413,17 @@ hgemm_status_t launch_stream(const CUtensorMap &ta, const CUtensorMap &tb, const
     attr_done[dev] = 1;
   }
   const uint32_t smem = p.stages * p.stage_bytes + 1024u /*align*/ + 512u /*barriers*/;
-  kern<<<static_cast<unsigned>(grid), 192, smem, stream>>>(ta, tb, p);
-  if (cudaPeekAtLastError() != cudaSuccess) return HGEMM_ERR_CUDA;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(static_cast<unsigned>(grid));
+  cfg.blockDim = dim3(192);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (cudaLaunchKernelEx(&cfg, kern, ta, tb, p) != cudaSuccess) return HGEMM_ERR_CUDA;
   g_launches.fetch_add(1, std::memory_order_relaxed);
   return HGEMM_SUCCESS;
 }

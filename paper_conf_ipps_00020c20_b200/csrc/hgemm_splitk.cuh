@@ -120,6 +120,7 @@ __global__ void __launch_bounds__(192, 1)
   } while (0)
 #endif
   if (threadIdx.x == 0) SK_TRACE(0);
+  griddep_wait();  // PDL: launch overlapped the previous kernel; C is read right below
   // Epilogue warps prefetch their C slice (FP16 vector path, beta != 0) at
   // kernel start: C does not depend on the accumulator.
   uint32_t cpre[SH::SLICE / 2];

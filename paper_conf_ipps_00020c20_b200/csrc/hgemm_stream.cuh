@@ -130,6 +130,7 @@ __global__ void __launch_bounds__(192, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  griddep_wait();  // PDL: the prologue overlapped the previous kernel
   if (threadIdx.x == 0) ST_TRACE(1);
 
   if (warp == 0) {

@@ -376,6 +376,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
   constexpr uint32_t A_KSTEP = A_MN ? 16 * 128 : 32;
   constexpr uint32_t B_KSTEP = B_MN ? 16 * 128 : 32;
 
+#ifdef HGEMM_TRACE
+  const unsigned long long cta_t0 = globaltimer_ns();  // kernel entry (before the prologue)
+#endif
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw_u32 = smem_u32(smem_raw);
   uint8_t *smem = smem_raw + ((1024u - (raw_u32 & 1023u)) & 1023u);
@@ -428,10 +431,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  griddep_wait();  // the prologue above overlapped the previous kernel; global memory from here on
   unsigned long long probe_clk = 0, probe_ns = 0;
-#ifdef HGEMM_TRACE
-  const unsigned long long cta_t0 = globaltimer_ns();
-#endif
+
   if (p.probe != nullptr && blockIdx.x == 0 && threadIdx.x == 0) {
     probe_clk = clock64();
     probe_ns = globaltimer_ns();
@@ -515,6 +517,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
         }
       }
+      griddep_launch_dependents();  // all loads issued: the next kernel may start its prologue
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (leader CTA)

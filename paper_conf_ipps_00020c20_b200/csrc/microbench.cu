@@ -239,7 +239,53 @@ EncodeTiledFn encode_fn() {
 }
 }  // namespace
 
+__global__ void stamp_kernel(unsigned long long *dst) {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  *dst = t;
+}
+
+__global__ void empty_kernel(unsigned long long *dst, int touch_smem) {
+  extern __shared__ uint8_t sm[];
+  if (touch_smem && threadIdx.x == 0) sm[0] = 1;
+  if (dst && threadIdx.x == 0 && blockIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    *dst = t;
+  }
+}
+
 extern "C" {
+
+// Empty kernel with the tile kernel's launch shape (grid, block, dynamic smem,
+// cluster size): the fixed cost of such a launch, nothing else.
+int mb_empty(int grid, int block, int smem, int cluster, unsigned long long *dst, cudaStream_t s) {
+  static int attr = 0;
+  if (!attr) {
+    if (cudaFuncSetAttribute(empty_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448) != cudaSuccess)
+      return 2;
+    attr = 1;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute a[1];
+  a[0].id = cudaLaunchAttributeClusterDimension;
+  a[0].val.clusterDim.x = cluster;
+  a[0].val.clusterDim.y = 1;
+  a[0].val.clusterDim.z = 1;
+  cfg.attrs = a;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, empty_kernel, dst, smem > 0 ? 1 : 0) == cudaSuccess ? 0 : 1;
+}
+
+// One-thread kernel writing %globaltimer to *dst (timeline probes around a launch).
+int mb_stamp(unsigned long long *dst, cudaStream_t s) {
+  stamp_kernel<<<1, 32, 0, s>>>(dst);
+  return cudaPeekAtLastError() == cudaSuccess ? 0 : 1;
+}
 
 // cycles[i] for CTA (or CTA pair) i; returns 0 on success.
 int mb_mma_rate(int cta_group, int n, int iters, int grid, int latency_mode, unsigned long long *cycles_dev) {

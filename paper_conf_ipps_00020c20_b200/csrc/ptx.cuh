@@ -370,6 +370,18 @@ __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t count) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
 }
 
+// ------------------------------------------------------------------ programmatic dependent launch
+// Kernels launched with cudaLaunchAttributeProgrammaticStreamSerialization may
+// start (barrier init, TMEM allocation, descriptor prefetch) while the previous
+// kernel of the stream drains; griddepcontrol.wait blocks until that kernel has
+// completed and its memory is visible, so it precedes every global access.
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+// Lets the next PDL kernel of the stream begin launching (its own wait still
+// orders its global accesses after this grid's completion).
+__device__ __forceinline__ void griddep_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // ------------------------------------------------------------------ cluster
 __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");

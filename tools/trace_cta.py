@@ -24,6 +24,7 @@ ap.add_argument("--beta", type=float, default=1.0)
 ap.add_argument("--kernel", default="auto")
 ap.add_argument("--bn", type=int, default=0)
 ap.add_argument("--sk", type=int, default=0)
+ap.add_argument("--warm", action="store_true", help="no L2 flush between launches")
 a = ap.parse_args()
 if a.kernel != "auto":
     binding.set_config(a.kernel, block_n=a.bn, stream_k=a.sk)
@@ -33,11 +34,18 @@ B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
 C = (torch.rand(n, m, device="cuda") * 2 - 1).half()
 flush = torch.empty(64 * 1024 * 1024, device="cuda")
 probe = torch.zeros(264 + 8 * 160, dtype=torch.int64, device="cuda")
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 for i in range(6):
-    flush.zero_()
+    if not a.warm:
+        flush.zero_()
     binding.set_probe(probe if i == 5 else None)
+    if i == 5:
+        e0.record()
     binding.hgemm(m, n, k, 1.0, A, k, B, k, a.beta, C, m, "T", "N", "f16")
+    if i == 5:
+        e1.record()
 torch.cuda.synchronize()
+print(f"event time of the probed launch: {e0.elapsed_time(e1) * 1e3:.1f} us")
 print(binding.get_stats())
 v = probe.cpu().view(-1).tolist()
 rows = [v[264 + 8 * b: 272 + 8 * b] for b in range(160) if v[264 + 8 * b]]
