@@ -279,11 +279,22 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
     if (p.probe != nullptr && blockIdx.x == 0 && (it) < 16)                              \
       p.probe[8 + 16 * (it) + (field)] = static_cast<unsigned long long>(clock64());     \
   } while (0)
-// Every CTA: %globaltimer of item `it` < 2 events at p.probe[264 + 8*blockIdx.x + 2 + 3*it + field].
+// Every CTA: %globaltimer at p.probe[264 + 8*blockIdx.x + slot]: 0 entry, 1 end,
+// 2 prologue done, 3 first TMA issued, 4 first full stage acquired (MMA leader),
+// 5 + field for the first work item: 5 MMA done, 6 epilogue wake, 7 epilogue done.
 #define HG_CTRACE(it, field)                                                             \
   do {                                                                                   \
-    if (p.probe != nullptr && (it) < 2)                                                  \
-      p.probe[264 + 8 * blockIdx.x + 2 + 3 * (it) + (field)] = globaltimer_ns();         \
+    if (p.probe != nullptr && (it) == 0)                                                 \
+      p.probe[264 + 8 * blockIdx.x + 5 + (field)] = globaltimer_ns();                   \
+  } while (0)
+#define HG_STAMP(slot)                                                                   \
+  do {                                                                                   \
+    if (p.probe != nullptr) p.probe[264 + 8 * blockIdx.x + (slot)] = globaltimer_ns();   \
+  } while (0)
+// second region (producer start-up detail): p.probe[264 + 8*160 + 8*blockIdx.x + slot]
+#define HG_STAMP2(slot)                                                                  \
+  do {                                                                                   \
+    if (p.probe != nullptr) p.probe[264 + 1280 + 8 * blockIdx.x + (slot)] = globaltimer_ns(); \
   } while (0)
 #else
 #define HG_TRACE(it, field) \
@@ -291,6 +302,12 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
   } while (0)
 #define HG_CTRACE(it, field) \
   do {                       \
+  } while (0)
+#define HG_STAMP(slot) \
+  do {                 \
+  } while (0)
+#define HG_STAMP2(slot) \
+  do {                  \
   } while (0)
 #endif
 
@@ -307,6 +324,7 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
 // and publishes each finished unit in its chunk's counter.  Units are taken from
 // a shared work index, so any subset of resident CTAs completes all of them.
 __device__ __forceinline__ void ag_copy_warp(const TcParams &p, uint32_t lane) {
+  griddep_wait();  // the work counters were zeroed by the previous operation of the stream
   const int64_t vpr = static_cast<int64_t>(p.K) / 8;  // 16-B vectors per row (K % 8 == 0)
   const int64_t ld_v = p.ag_lda / 8;
   for (;;) {
@@ -388,7 +406,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
   uint64_t *tfull = empty + STAGES;      // [ACC][NH]
   uint64_t *tempty = tfull + ACC * NH;   // [ACC][NH]
   uint64_t *skbar = tempty + ACC * NH;   // [EPI_WARPS][2]: stream-K partial loads
-  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(skbar + 2 * S::EPI_WARPS);
+  uint64_t *cgo = skbar + 2 * S::EPI_WARPS;  // the first stages are issued: C loads may start
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(cgo + 1);
 
   const uint32_t warp = warp_id();
   const uint32_t lane = lane_id();
@@ -422,6 +441,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         }
       }
       for (int b = 0; b < 2 * S::EPI_WARPS; ++b) mbar_init(&skbar[b], 1);
+      mbar_init(cgo, 1);
       fence_mbarrier_init();
     }
     __syncwarp();
@@ -431,7 +451,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  griddep_wait();  // the prologue above overlapped the previous kernel; global memory from here on
+  // Programmatic dependent launch: everything above overlapped the previous kernel
+  // of the stream.  Each role calls griddep_wait() before its first global memory
+  // access (the producer after computing its first tile, the epilogue before C, the
+  // copy warp before the peers); the MMA warp touches only shared memory and TMEM.
   unsigned long long probe_clk = 0, probe_ns = 0;
 
   if (p.probe != nullptr && blockIdx.x == 0 && threadIdx.x == 0) {
@@ -448,9 +471,16 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       const uint64_t pol_b = p.l2_hint == 1 ? l2_policy_evict_first() : p.l2_hint == 2 ? l2_policy_evict_normal() : 0;
       uint32_t stage = 0, phase = 0;
       WorkItem wi;
+      HG_STAMP2(0);
+      bool cgo_sent = false;
       for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i) {
         int tm, tn;
         tile_coords(wi.tile, p, tm, tn);
+        if (i == 0) {
+          HG_STAMP2(1);
+          griddep_wait();  // first global access of this role below
+          HG_STAMP(2);
+        }
         const int a_row = (tm * MC + static_cast<int>(pair)) * BM * CG + static_cast<int>(prank) * BM;
         const int b_row0 = tn * BN + static_cast<int>(prank) * B_ROWS;
         if constexpr (AG) {
@@ -468,6 +498,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         }
         for (int kb = wi.kb0; kb < wi.kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1u);
+#ifdef HGEMM_TRACE
+          if (i == 0 && kb == wi.kb0) HG_STAMP2(2);
+#endif
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
           const uint32_t sb = sa + A_BYTES;
           uint32_t fb;
@@ -479,9 +512,15 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             fb = mapa_shared(smem_u32(&full[stage]), leader);
           }
           const int k0 = kb * BK;
+#ifdef HGEMM_TRACE
+          if (i == 0 && kb == wi.kb0) HG_STAMP2(3);
+#endif
           if constexpr (!A_MN) {
             if constexpr (CG == 1) tma_load_2d(&tmA, sa, fb, k0, a_row, pol_a);
             else tma_load_2d_pair(&tmA, sa, fb, k0, a_row, pol_a);
+#ifdef HGEMM_TRACE
+            if (i == 0 && kb == wi.kb0) HG_STAMP2(4);
+#endif
           } else {
 #pragma unroll
             for (int q = 0; q < BM / 64; ++q) {
@@ -514,9 +553,19 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
               }
             }
           }
+#ifdef HGEMM_TRACE
+          if (i == 0 && kb == wi.kb0) HG_STAMP(3);
+#endif
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+          // the first ring's worth of operand loads is queued: the epilogue's C loads
+          // (beta != 0) may follow without delaying the start of the mainloop
+          if (!cgo_sent && (i > 0 || kb + 1 - wi.kb0 >= STAGES || kb + 1 == wi.kb1)) {
+            mbar_arrive(cgo);
+            cgo_sent = true;
+          }
         }
       }
+      if (!cgo_sent) mbar_arrive(cgo);
       griddep_launch_dependents();  // all loads issued: the next kernel may start its prologue
     }
   } else if (warp == 1) {
@@ -593,6 +642,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           tc_fence_after();
           if (kb == 0) {
             HG_TRACE(it, 6);
+            if (it == 0) HG_STAMP(4);
             // accumulator half 0 must have been drained by the previous tile's epilogue
             if constexpr (CG == 2) mbar_wait_cluster(&tempty[buf * NH], acc_phase ^ 1u);
             else mbar_wait(&tempty[buf * NH], acc_phase ^ 1u);
@@ -647,6 +697,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
     if constexpr (AG) ag_copy_warp(p, lane);
   } else {
     // ------------------------------------------------------------ epilogue warps
+    griddep_wait();  // C may be read (beta != 0) and D is written below
     const uint32_t quad = warp & 3u;                 // TMEM lane quadrant this warp may access
     const uint32_t ew = warp - 2u;                   // epilogue warp index 0..7
     const int cgrp = static_cast<int>(ew >> 2);      // which half of each accumulator half's columns
@@ -719,6 +770,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         tma_load_2d(&tmD, stg + b * (32u * 128u), smem_u32(&skbar[ew * 2 + b]), box_col(j), row_base, 0);
       };
       if (c_tma && lane == 0) {
+        if (it == 0) mbar_wait(cgo, 0);  // behind the first operand stages in the memory queues
         bulk_wait_group_read<0>();  // earlier stores have read every staging box of this warp
 #pragma unroll
         for (int j = 0; j < NBT; ++j) {
@@ -1020,7 +1072,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         }
       }
     }
-    if (lane == 0) bulk_wait_group<0>();
+    // the staging buffers must have been read before the CTA exits; the stores'
+    // global writes complete with the grid (the next kernel's griddepcontrol.wait
+    // or stream order sees them)
+    if (lane == 0) bulk_wait_group_read<0>();
   }
 
   // Reconverge each warp (the role code ran on one lane of warps 0/1) before the
