@@ -331,9 +331,11 @@ __global__ void __launch_bounds__(192, 1)
   }
 
   if (threadIdx.x == 64) SK_TRACE(6);
-  // peers must not exit while their shared memory is being read
-  __syncwarp();  // reconverge the single-lane roles before the .aligned cluster barrier
-  cluster_sync();
+  // No second cluster barrier: every remote (DSMEM) access of this kernel is a push
+  // that completed before the barrier above; the reduction reads local shared
+  // memory only, so a CTA may exit without waiting for its peers.
+  __syncwarp();
+  __syncthreads();
   if (threadIdx.x == 0) SK_TRACE(7);
   if (warp == 1) {
     tc_fence_after();
