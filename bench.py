@@ -60,46 +60,64 @@ def load_traffic(workload):
 
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
-    """Samples SM clock and throttle reasons during the timed region (nvidia-smi, else NVML)."""
+    """Samples SM clock and throttle reasons during the timed region (NVML).
+
+    NVML is initialised and sampled once in start(), before the timed region
+    begins, and once more in stop(), so even a region shorter than the sampling
+    period carries samples taken around and inside it."""
 
     def __init__(self, index=0):
         self.index = index
         self.samples = []
         self._stop = threading.Event()
         self._t = None
+        self._h = None
 
-    def _nvml_loop(self):
+    def _sample(self):
+        import pynvml
+        h = self._h
+        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+        try:
+            rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+        except Exception:
+            rs = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+        self.samples.append((sm, self._max, [k for k, v in self._names.items() if rs & v]))
+
+    def _loop(self):
+        try:
+            while not self._stop.wait(0.005):
+                self._sample()
+        except Exception as e:  # pragma: no cover
+            self.samples.append((None, None, [f"nvml-error:{type(e).__name__}"]))
+
+    def start(self):
         try:
             import pynvml
             pynvml.nvmlInit()
-            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
-            mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
-            names = {
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self._max = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+            self._names = {
                 "hw_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwSlowdown", 0x8),
                 "hw_thermal_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
                 "sw_thermal_slowdown": getattr(pynvml, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
                 "sw_power_cap": getattr(pynvml, "nvmlClocksEventReasonSwPowerCap", 0x4),
                 "hw_power_brake_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
             }
-            while not self._stop.is_set():
-                sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
-                try:
-                    rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
-                except Exception:
-                    rs = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h)
-                self.samples.append((sm, mx, [k for k, v in names.items() if rs & v]))
-                time.sleep(0.01)
+            self._sample()
         except Exception as e:  # pragma: no cover
             self.samples.append((None, None, [f"nvml-error:{type(e).__name__}"]))
-
-    def start(self):
-        self._t = threading.Thread(target=self._nvml_loop, daemon=True)
+            return
+        self._t = threading.Thread(target=self._loop, daemon=True)
         self._t.start()
 
     def stop(self):
         self._stop.set()
         if self._t:
             self._t.join(timeout=2)
+            try:
+                self._sample()
+            except Exception:  # pragma: no cover
+                pass
         sm = [s[0] for s in self.samples if s[0]]
         reasons = sorted({r for s in self.samples for r in s[2]})
         return {"sm_mhz": statistics.median(sm) if sm else None,
