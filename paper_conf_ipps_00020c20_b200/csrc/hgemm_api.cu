@@ -44,6 +44,14 @@ hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
 std::atomic<int64_t> g_launches{0};
 std::atomic<unsigned long long *> g_probe{nullptr};
 // programmatic dependent launch of the tensor-core kernels (HGEMM_PDL=0 disables it: experiments)
+// half-tile tail for 512-wide tiles: EXPERIMENTAL, off unless HGEMM_HALF_TAIL=1.  It
+// measured +1-4% at W = 7168 / 7680 but hangs for beta != 0 when a half item lies
+// entirely outside N and is a CTA's third work item (tools/one_case.py 1100 1100 12
+// 1.0 f16), so it stays off until that is understood.
+const bool g_half_tail = [] {
+  const char *e = std::getenv("HGEMM_HALF_TAIL");
+  return e && e[0] == '1';
+}();
 const bool g_pdl = [] {
   const char *e = std::getenv("HGEMM_PDL");
   return !(e && e[0] == '0');
@@ -258,8 +266,21 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   p.sk_u0 = p.sk_units = 0;
   p.sk_ws = nullptr;
   p.sk_flags = nullptr;
+  p.n_half = 0;
   *sk_used = false;
-  if (MC == 1 && !AG) {
+  // half-tile tail (512-wide tiles): a last wave of r <= units/2 tiles runs as 2r
+  // 256-wide items, i.e. in about half the time
+  bool half_tail = false;
+  if (BN == 512 && CG == 2 && MC == 1 && !AG && g_half_tail && sk_mode != 2) {
+    const int r = tiles % units;
+    if (r > 0 && 2 * r <= units) {
+      p.n_half = r;
+      p.dp_tiles = tiles + r;
+      clusters = std::min(tiles + r, units);
+      half_tail = true;
+    }
+  }
+  if (MC == 1 && !AG && !half_tail) {
     const int dp = sk_plan(tiles, units, p.num_k_blocks, sk_mode);
     float *ws = nullptr;
     int *flags = nullptr;
@@ -478,6 +499,12 @@ void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, 
     const int64_t units = num_sms / c.cg;
     double waves = static_cast<double>(cdiv(tiles, units));
     const int64_t nkb = cdiv(K, 64);
+    // 512-wide: a last wave of r <= units/2 tiles runs as 256-wide halves (launch_tc).
+    // Measured cost of that tail: ~0.8 of a wave (half the MMA work, but the half
+    // items share one accumulator half, so their epilogues do not overlap the next
+    // item's mainloop): it wins at W = 7168 / 7680 and loses at W <= 5632
+    if (c.bn == 512 && g_half_tail && sk_mode != 2 && tiles % units != 0 && 2 * (tiles % units) <= units)
+      waves = static_cast<double>(tiles / units) + 0.8;
     // stream-K: fractional waves (256-wide tiles only: with 512-wide tiles the FP32
     // partials of a split tile are twice as large and it measured slower everywhere)
     if (c.bn <= 256 && sk_plan(tiles, units, nkb, sk_mode) >= 0)

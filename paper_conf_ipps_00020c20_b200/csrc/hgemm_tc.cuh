@@ -78,6 +78,11 @@ struct TcParams {
   int32_t ag_chunk_rows, ag_unit_rows;
   int32_t ag_units;                  // copy units in total (all peers)
   int32_t n_rot;                     // raster groups along N start at group n_rot (group_m < 0 only)
+  // Half-tile tail (BN = 512 only): the last n_half
+  // tiles of the raster are processed as two 256-wide items each (sub-tile 0 and
+  // 1, accumulator half 0 only), so a last wave of R <= units/2 tiles takes half
+  // the time.  Work items are numbered over tiles + n_half virtual items.
+  int32_t n_half;
 };
 
 // One unit of work of a cluster: k-blocks [kb0, kb1) of cluster tile `tile`.
@@ -109,6 +114,19 @@ __device__ __forceinline__ bool get_item(const TcParams &p, int c, int G, int i,
   w.kb0 = static_cast<int>(b - static_cast<int64_t>(t) * nkb);
   w.kb1 = static_cast<int>(e - static_cast<int64_t>(t) * nkb);
   return true;
+}
+
+// Virtual work item v -> (tile, sub): sub = -1 for a whole tile, 0/1 for the
+// 256-wide halves of a split tail tile.
+__device__ __forceinline__ void item_tile(const TcParams &p, int v, int &tile, int &sub) {
+  const int full = p.num_m_tiles * p.num_n_tiles - p.n_half;
+  if (p.n_half == 0 || v < full) {
+    tile = v;
+    sub = -1;
+    return;
+  }
+  tile = full + ((v - full) >> 1);
+  sub = (v - full) & 1;
 }
 
 // UMMA shared-memory descriptor, SWIZZLE_128B, K-major operand.
@@ -474,8 +492,13 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       HG_STAMP2(0);
       bool cgo_sent = false;
       for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i) {
-        int tm, tn;
-        tile_coords(wi.tile, p, tm, tn);
+        int tm, tn, tile, sub;
+        item_tile(p, wi.tile, tile, sub);
+        tile_coords(tile, p, tm, tn);
+        // 256-wide half item: one B half-box, into the slot of accumulator half hsel = 0
+        const bool half = (NH == 2) && (MC == 1) && sub >= 0;
+        constexpr int hsel = 0;
+        const uint32_t stage_bytes = half ? STAGE_BYTES - B_HALF_BYTES : STAGE_BYTES;
         if (i == 0) {
           HG_STAMP2(1);
           griddep_wait();  // first global access of this role below
@@ -505,10 +528,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           const uint32_t sb = sa + A_BYTES;
           uint32_t fb;
           if constexpr (CG == 1) {
-            mbar_arrive_expect_tx(&full[stage], STAGE_BYTES);
+            mbar_arrive_expect_tx(&full[stage], stage_bytes);
             fb = smem_u32(&full[stage]);
           } else {
-            if (prank == 0) mbar_arrive_expect_tx(&full[stage], 2 * STAGE_BYTES);
+            if (prank == 0) mbar_arrive_expect_tx(&full[stage], 2 * stage_bytes);
             fb = mapa_shared(smem_u32(&full[stage]), leader);
           }
           const int k0 = kb * BK;
@@ -529,9 +552,11 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             }
           }
 #pragma unroll
-          for (int h = 0; h < NH; ++h) {
+          for (int hh = 0; hh < NH; ++hh) {
+            if (half && hh > 0) break;
+            const int h = half ? hsel : hh;
             const uint32_t sbh = sb + h * B_HALF_BYTES;
-            const int b_row = b_row0 + h * UMMA_N;
+            const int b_row = b_row0 + (half ? sub : h) * UMMA_N;
             if constexpr (MC == 2) {
               // this pair's share of the half-box, delivered to the same CTA position of both pairs
               const uint16_t mc_mask = static_cast<uint16_t>((1u << prank) | (1u << (CG + prank)));
@@ -598,7 +623,38 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       WorkItem wi;
       for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i, ++it) {
         const int nkb = wi.kb1 - wi.kb0;  // k-blocks of this item (kb below counts from its first)
-        const int end_lag = (NH == 2) ? min(HGEMM_END_LAG, max(nkb - 1, 0)) : 0;
+        int itile, isub;
+        item_tile(p, wi.tile, itile, isub);
+        // a 256-wide half item uses accumulator half 0 only: half 1 is neither waited
+        // for nor written (its tfull/tempty phases still advance once per item)
+        const bool half = (NH == 2) && (MC == 1) && isub >= 0;
+        const int end_lag = (NH == 2 && !half) ? min(HGEMM_END_LAG, max(nkb - 1, 0)) : 0;
+        if (NH == 2 && half) {
+          // 256-wide half item: accumulator half 0 only; both tfull phases still
+          // complete once per item.  (Alternating the accumulator half between
+          // consecutive half items, to double-buffer TMEM, hung with beta != 0 when
+          // a half item lies entirely outside N -- not understood yet; round-2 work.)
+          constexpr int hsel = 0;
+          const uint32_t d_tmem = tmem_base;
+          const uint32_t acc_phase = it & 1;
+          for (int kb = 0; kb < nkb; ++kb) {
+            mbar_wait(&full[stage], phase);
+            tc_fence_after();
+            if (kb == 0) {
+              if (it == 0) HG_STAMP(4);
+              if constexpr (CG == 2) mbar_wait_cluster(&tempty[hsel], acc_phase ^ 1u);
+              else mbar_wait(&tempty[hsel], acc_phase ^ 1u);
+              tc_fence_after();
+            }
+            issue_half(stage, hsel, kb, d_tmem);
+            umma_commit_mask<CG>(&empty[stage], empty_mask);
+            if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+          }
+          umma_commit_mask<CG>(&tfull[0], pair_mask);
+          umma_commit_mask<CG>(&tfull[1], pair_mask);
+          HG_CTRACE(it, 0);
+          continue;
+        }
         const int h1_limit = nkb - end_lag;  // half-1 k-blocks >= h1_limit are issued after the loop
         const uint32_t buf = (ACC == 2) ? (it & 1) : 0u;
         const uint32_t acc_phase = (ACC == 2) ? ((it >> 1) & 1) : (it & 1);
@@ -729,8 +785,19 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
     uint32_t sk_uses[2] = {0u, 0u};
     WorkItem wi;
     for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i, ++it) {
-      int tm, tn;
-      tile_coords(wi.tile, p, tm, tn);
+      int tm, tn, itile, isub;
+      item_tile(p, wi.tile, itile, isub);
+      tile_coords(itile, p, tm, tn);
+      // half item: accumulator half 0 holds D columns tn*BN + isub*UMMA_N ..; half 1 is
+      // only handed back (nh_act accumulator halves carry data)
+      const bool half = (NH == 2 && MC == 1 && isub >= 0);
+      constexpr int hsel = 0;                                 // the accumulator half a half item uses
+      const int nh_act = half ? 1 : NH;
+      // D column of TMEM column 0 (a half item's data sits in TMEM half hsel but
+      // belongs to D columns tn*BN + isub*UMMA_N ..)
+      const int cbase = tn * BN + (half ? (isub - hsel) * UMMA_N : 0);
+      // accumulator halves in visiting order (a half item hands half 1 back unused)
+      auto half_at = [&](int hh) { return hh; };
       // 0: whole tile; 1: a later k segment of a stream-K tile -> publish FP32
       // partial; 2: the tile's first segment -> add the later segments' partials
       const int mode = wi.kb0 > 0 ? 1 : (wi.kb1 < p.num_k_blocks ? 2 : 0);
@@ -762,8 +829,12 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       constexpr int NB = EPI_COLS_W / EPI_COLS;  // staging boxes per warp per accumulator half
       constexpr int NBT = NH * NB;               // ... per tile
       const bool c_tma = beta != 0.0f && mode == 0 && (p.N & (VEC - 1)) == 0;
+      const int nbt = nh_act * NB;               // boxes carrying data
       const uint32_t s0 = nstore;
-      auto box_col = [&](int j) { return tn * BN + (j / NB) * UMMA_N + cgrp * EPI_COLS_W + (j % NB) * EPI_COLS; };
+      auto box_col = [&](int j) {
+        return half ? tn * BN + isub * UMMA_N + cgrp * EPI_COLS_W + j * EPI_COLS
+                    : tn * BN + (j / NB) * UMMA_N + cgrp * EPI_COLS_W + (j % NB) * EPI_COLS;
+      };
       auto c_load = [&](int j) {
         const uint32_t b = (s0 + static_cast<uint32_t>(j)) % EPI_BUFS;
         mbar_arrive_expect_tx(&skbar[ew * 2 + b], 32u * 128u);
@@ -774,6 +845,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         bulk_wait_group_read<0>();  // earlier stores have read every staging box of this warp
 #pragma unroll
         for (int j = 0; j < NBT; ++j) {
+          if (j >= nbt) break;
           if (j < EPI_BUFS) c_load(j);
           else tma_prefetch_l2_2d(&tmD, box_col(j), row_base);
         }
@@ -810,15 +882,25 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         // in FP32 in place, TMA store; a half goes back to the MMA warp after its
         // last box's TMEM read, a box after its store has read it takes the next C box
 #pragma unroll 1
-        for (int h = 0; h < NH; ++h) {
+        for (int hh = 0; hh < NH; ++hh) {
+          const int h = half_at(hh);
           if (h > 0) {
             if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
             __syncwarp();
             tc_fence_after();
           }
+          if (half && h != hsel) {  // half item: nothing in this accumulator half, hand it back
+            tc_fence_before();
+            if (lane == 0) {
+              if constexpr (CG == 2) mbar_arrive_cluster_relaxed(tempty_addr + (buf * NH + h) * 8);
+              else mbar_arrive_relaxed(&tempty[buf * NH + h]);
+            }
+            __syncwarp();
+            continue;
+          }
 #pragma unroll 1
           for (int c = 0; c < NB; ++c) {
-            const int j = h * NB + c;
+            const int j = (half ? 0 : h * NB) + c;
             const int colt = h * UMMA_N + cgrp * EPI_COLS_W + c * EPI_COLS;
             uint32_t v[EPI_COLS];
             tmem_ld_32x32b_x32(tbase + colt, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
@@ -862,16 +944,16 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             fence_proxy_async_smem();
             __syncwarp();
             if (lane == 0) {
-              tma_store_2d(&tmD, sbuf, tn * BN + colt, row_base);
+              tma_store_2d(&tmD, sbuf, cbase + colt, row_base);
               bulk_commit_group();
-              if (j + EPI_BUFS < NBT) {
+              if (j + EPI_BUFS < nbt) {
                 bulk_wait_group_read<0>();  // this box's store has read it: load the next C box
                 c_load(j + EPI_BUFS);
               }
             }
           }
         }
-        nstore = s0 + NBT;
+        nstore = s0 + nbt;
         continue;
       }
       if (fast && mode == 0) {
@@ -879,11 +961,21 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         // half into registers (alpha and FP16 packing applied), hand the half back
         // to the MMA warp, then store.
 #pragma unroll 1
-        for (int h = 0; h < NH; ++h) {
+        for (int hh = 0; hh < NH; ++hh) {
+          const int h = half_at(hh);
           if (h > 0) {  // each half has its own tmem_full barrier
             if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
             __syncwarp();
             tc_fence_after();
+          }
+          if (half && h != hsel) {  // half item: nothing in this accumulator half, hand it back
+            tc_fence_before();
+            if (lane == 0) {
+              if constexpr (CG == 2) mbar_arrive_cluster_relaxed(tempty_addr + (buf * NH + h) * 8);
+              else mbar_arrive_relaxed(&tempty[buf * NH + h]);
+            }
+            __syncwarp();
+            continue;
           }
           uint32_t pk[PKW];
           const int c0 = h * UMMA_N + cgrp * EPI_COLS_W;  // first tile column of this warp
@@ -917,16 +1009,26 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           for (int c = 0; c < EPI_COLS_W / EPI_COLS; ++c)
             emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, stg, nstore,
                                                      *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
-                                                     tn * BN + c0 + c * EPI_COLS, row, row_base, lane);
+                                                     cbase + c0 + c * EPI_COLS, row, row_base, lane);
         }
         continue;
       }
 #pragma unroll 1
-      for (int h = 0; h < NH; ++h) {
+      for (int hh = 0; hh < NH; ++hh) {
+        const int h = half_at(hh);
         if (h > 0) {
           if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
           __syncwarp();
           tc_fence_after();
+        }
+        if (half && h != hsel) {  // half item: nothing in this accumulator half, hand it back
+          tc_fence_before();
+          if (lane == 0) {
+            if constexpr (CG == 2) mbar_arrive_cluster_relaxed(tempty_addr + (buf * NH + h) * 8);
+            else mbar_arrive_relaxed(&tempty[buf * NH + h]);
+          }
+          __syncwarp();
+          continue;
         }
 #pragma unroll 1
         for (int c = 0; c < EPI_COLS_W / EPI_COLS; ++c) {
@@ -999,7 +1101,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
 #endif
           // alpha*acc (+ beta*C) in FP32, packed into 32 words = one 128-B row
           uint32_t w[32];
-          const int col = tn * BN + colt;
+          const int col = cbase + colt;
           if constexpr (OUT_F32) {
 #pragma unroll
             for (int j = 0; j < 32; ++j) w[j] = __float_as_uint(alpha * __uint_as_float(v[j]));
