@@ -124,6 +124,11 @@ typedef struct {
                           a tile split between clusters is summed in k order through a library-owned
                           FP32 workspace (per device and stream, allocated on first use, never during
                           stream capture), so results are deterministic for a given device. */
+    int32_t half_tail; /* 512-wide 2-SM tiles: 0 = auto (when r tiles are left for a last wave after
+                          at least 4 whole waves and r <= clusters/2, those r tiles are processed as
+                          2r 256-wide items), 1 = never, 2 = whenever r <= clusters/2.  Same per-element
+                          arithmetic as whole tiles.  hgemm_get_last_config reports 2 if it was used,
+                          1 if not (tile kernels). */
 } hgemm_config_t;
 
 /* Set (cfg != NULL) or reset to automatic (cfg == NULL) the process-global

@@ -39,19 +39,12 @@ constexpr int kMaxDevices = 64;
 DeviceInfo g_dev[kMaxDevices];
 std::mutex g_mu;
 
-hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
-hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
+hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0};
+hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0};
 std::atomic<int64_t> g_launches{0};
 std::atomic<unsigned long long *> g_probe{nullptr};
 // programmatic dependent launch of the tensor-core kernels (HGEMM_PDL=0 disables it: experiments)
-// half-tile tail for 512-wide tiles: EXPERIMENTAL, off unless HGEMM_HALF_TAIL=1.  It
-// measured +1-4% at W = 7168 / 7680 but hangs for beta != 0 when a half item lies
-// entirely outside N and is a CTA's third work item (tools/one_case.py 1100 1100 12
-// 1.0 f16), so it stays off until that is understood.
-const bool g_half_tail = [] {
-  const char *e = std::getenv("HGEMM_HALF_TAIL");
-  return e && e[0] == '1';
-}();
+thread_local bool t_half_used = false;  // the last tile launch of this thread used the half-tile tail
 const bool g_pdl = [] {
   const char *e = std::getenv("HGEMM_PDL");
   return !(e && e[0] == '0');
@@ -231,6 +224,8 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
                          cudaStream_t stream) {
   using S = TcShape<BN, CG, OUT_F32>;
   constexpr int THREADS = S::THREADS + (AG ? 32 : 0);  // + the all-gather copy warp
+  const int ht_mode = sk_mode >> 4;  // hgemm_config_t::half_tail, packed above the stream-K mode
+  sk_mode &= 15;
   auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC, AG>;
   static int attr_done[kMaxDevices] = {};
   static int max_clusters[kMaxDevices] = {};
@@ -271,15 +266,16 @@ hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUt
   // half-tile tail (512-wide tiles): a last wave of r <= units/2 tiles runs as 2r
   // 256-wide items, i.e. in about half the time
   bool half_tail = false;
-  if (BN == 512 && CG == 2 && MC == 1 && !AG && g_half_tail && sk_mode != 2) {
+  if (BN == 512 && CG == 2 && MC == 1 && !AG && ht_mode != 1 && sk_mode != 2) {
     const int r = tiles % units;
-    if (r > 0 && 2 * r <= units) {
+    if (r > 0 && 2 * r <= units && (ht_mode == 2 || tiles / units >= 4)) {
       p.n_half = r;
       p.dp_tiles = tiles + r;
       clusters = std::min(tiles + r, units);
       half_tail = true;
     }
   }
+  t_half_used = half_tail;
   if (MC == 1 && !AG && !half_tail) {
     const int dp = sk_plan(tiles, units, p.num_k_blocks, sk_mode);
     float *ws = nullptr;
@@ -499,15 +495,15 @@ void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, 
     const int64_t units = num_sms / c.cg;
     double waves = static_cast<double>(cdiv(tiles, units));
     const int64_t nkb = cdiv(K, 64);
-    // 512-wide: a last wave of r <= units/2 tiles runs as 256-wide halves (launch_tc).
-    // Measured cost of that tail: ~0.8 of a wave (half the MMA work, but the half
-    // items share one accumulator half, so their epilogues do not overlap the next
-    // item's mainloop): it wins at W = 7168 / 7680 and loses at W <= 5632
-    if (c.bn == 512 && g_half_tail && sk_mode != 2 && tiles % units != 0 && 2 * (tiles % units) <= units)
-      waves = static_cast<double>(tiles / units) + 0.8;
+    // 512-wide: a last wave of r <= units/2 tiles after >= 4 whole waves runs as
+    // 256-wide halves (launch_tc), measured ~0.6 of a wave
+    const int ht_mode = sk_mode >> 4;
+    if (c.bn == 512 && ht_mode != 1 && (sk_mode & 15) != 2 && tiles % units != 0 &&
+        2 * (tiles % units) <= units && (ht_mode == 2 || tiles / units >= 4))
+      waves = static_cast<double>(tiles / units) + 0.6;
     // stream-K: fractional waves (256-wide tiles only: with 512-wide tiles the FP32
     // partials of a split tile are twice as large and it measured slower everywhere)
-    if (c.bn <= 256 && sk_plan(tiles, units, nkb, sk_mode) >= 0)
+    if (c.bn <= 256 && sk_plan(tiles, units, nkb, sk_mode & 15) >= 0)
       waves = static_cast<double>(tiles) / units + sk_overhead_waves(nkb);
     const double t = waves * (128.0 * c.cg * c.bn) / (c.cg * eff);
     if (t < best * 0.999) { best = t; cg = c.cg; bn = c.bn; }
@@ -531,11 +527,12 @@ const char *hgemm_status_string(hgemm_status_t s) {
 hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!cfg) {
-    g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0};
+    g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0};
     return HGEMM_SUCCESS;
   }
   if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_STREAM) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->stream_k < 0 || cfg->stream_k > 2) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->half_tail < 0 || cfg->half_tail > 2) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_SPLITK) {
     if (cfg->block_n != 0 && cfg->block_n != 64 && cfg->block_n != 128) return HGEMM_ERR_INVALID_VALUE;
     if (cfg->splits != 0 && cfg->splits != 2 && cfg->splits != 4 && cfg->splits != 8) return HGEMM_ERR_INVALID_VALUE;
@@ -754,7 +751,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   // the fused all-gather kernels exist for CTA pairs only
   const int forced_cg = ag ? 2 : cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
   // stream-K is off under the fused all-gather (its work items do not follow the chunk order)
-  const int skm = ag ? 1 : cfg.stream_k;
+  // stream-K mode with hgemm_config_t::half_tail packed above it (launch_tc, choose_tc)
+  const int skm = (ag ? 1 : cfg.stream_k) | (cfg.half_tail << 4);
   if (forced_cg && cfg.block_n && !(ag && cfg.block_n == 128)) { cg = forced_cg; bn = cfg.block_n; }
   else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, skm, cg, bn);
   const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
@@ -847,7 +845,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     st = dispatch_tc_layout<128, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);
-    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0, sk_used ? 2 : 1};
+    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0, sk_used ? 2 : 1,
+              t_half_used ? 2 : 1};
   }
   return st;
 }

@@ -495,9 +495,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         int tm, tn, tile, sub;
         item_tile(p, wi.tile, tile, sub);
         tile_coords(tile, p, tm, tn);
-        // 256-wide half item: one B half-box, into the slot of accumulator half hsel = 0
+        // 256-wide half item: one B half-box, into the slot of accumulator half hsel
+        // (alternating per item, so consecutive half items double-buffer TMEM)
         const bool half = (NH == 2) && (MC == 1) && sub >= 0;
-        constexpr int hsel = 0;
+        const int hsel = i & 1;
         const uint32_t stage_bytes = half ? STAGE_BYTES - B_HALF_BYTES : STAGE_BYTES;
         if (i == 0) {
           HG_STAMP2(1);
@@ -630,11 +631,14 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         const bool half = (NH == 2) && (MC == 1) && isub >= 0;
         const int end_lag = (NH == 2 && !half) ? min(HGEMM_END_LAG, max(nkb - 1, 0)) : 0;
         if (NH == 2 && half) {
-          // 256-wide half item: accumulator half 0 only; both tfull phases still
-          // complete once per item.  (Alternating the accumulator half between
-          // consecutive half items, to double-buffer TMEM, hung with beta != 0 when
-          // a half item lies entirely outside N -- not understood yet; round-2 work.)
-          constexpr int hsel = 0;
+          // 256-wide half item: accumulator half hsel only (alternating per item, so
+          // consecutive half items double-buffer TMEM); both tfull phases still
+          // complete once per item.  Before committing tfull[h] of this item the
+          // MMA warp must have observed tempty[h] of the previous item, for BOTH
+          // halves: otherwise it could complete two tfull phases of the unused half
+          // before the epilogue waited for the first, and the parity wait would
+          // alias (observed as a hang with a slow beta != 0 epilogue).
+          const int hsel = it & 1;
           const uint32_t d_tmem = tmem_base;
           const uint32_t acc_phase = it & 1;
           for (int kb = 0; kb < nkb; ++kb) {
@@ -650,6 +654,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             umma_commit_mask<CG>(&empty[stage], empty_mask);
             if (++stage == STAGES) { stage = 0; phase ^= 1u; }
           }
+          if constexpr (CG == 2) mbar_wait_cluster(&tempty[1 - hsel], acc_phase ^ 1u);
+          else mbar_wait(&tempty[1 - hsel], acc_phase ^ 1u);
           umma_commit_mask<CG>(&tfull[0], pair_mask);
           umma_commit_mask<CG>(&tfull[1], pair_mask);
           HG_CTRACE(it, 0);
@@ -791,13 +797,13 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       // half item: accumulator half 0 holds D columns tn*BN + isub*UMMA_N ..; half 1 is
       // only handed back (nh_act accumulator halves carry data)
       const bool half = (NH == 2 && MC == 1 && isub >= 0);
-      constexpr int hsel = 0;                                 // the accumulator half a half item uses
+      const int hsel = it & 1;                                // the accumulator half a half item uses
       const int nh_act = half ? 1 : NH;
       // D column of TMEM column 0 (a half item's data sits in TMEM half hsel but
       // belongs to D columns tn*BN + isub*UMMA_N ..)
       const int cbase = tn * BN + (half ? (isub - hsel) * UMMA_N : 0);
-      // accumulator halves in visiting order (a half item hands half 1 back unused)
-      auto half_at = [&](int hh) { return hh; };
+      // accumulator halves in visiting order: a half item hands its unused half back first
+      auto half_at = [&](int hh) { return half ? (hh == 0 ? 1 - hsel : hsel) : hh; };
       // 0: whole tile; 1: a later k segment of a stream-K tile -> publish FP32
       // partial; 2: the tile's first segment -> add the later segments' partials
       const int mode = wi.kb0 > 0 ? 1 : (wi.kb1 < p.num_k_blocks ? 2 : 0);

@@ -455,18 +455,16 @@ def test_stream_kernel_auto_and_fallback(oracle_mod):
         assert np.all(np.abs(g - r) <= 1e-3 * ab + ulp16(np.maximum(np.abs(g), np.abs(r))))
 
 
-# Half-tile tail (experimental, enabled with
-# HGEMM_HALF_TAIL=1 in the environment of the test process, otherwise these cases
-# run the plain 512-wide path): with 512-wide tiles, a last wave of
-# r <= clusters/2 tiles runs as 2r 256-wide items.  (m, n, max_ctas): kernel tiles =
+# Half-tile tail (forced with hgemm_config_t.half_tail = 2):
+# with 512-wide tiles, a last wave of r <= clusters/2 tiles runs as 2r 256-wide items.  (m, n, max_ctas): kernel tiles =
 # ceil(n/256) x ceil(m/512); clusters = max_ctas/2.
 #   (1500, 1100, 12): 5 x 3 = 15 tiles on 6 clusters -> 2 whole waves + 3 split tiles
 #   (1100, 1100, 12): same grid, the last tile column is 76 wide: its second half is
 #                     entirely outside N (loads zero-filled, stores clipped)
 #   (1100,  700,  0): 3 x 3 = 9 tiles on 74 clusters -> every tile split
-#   (1497, 1100, 16): 15 tiles on 8 clusters -> 1 wave + 7 split tiles; N = 1497 is
+#   (1497, 1100, 22): 15 tiles on 11 clusters -> 1 wave + 4 split tiles; N = 1497 is
 #                     not a multiple of 16 B -> chunked epilogue
-HALF_CASES = [(1500, 1100, 12), (1100, 1100, 12), (1100, 700, 0), (1497, 1100, 16)]
+HALF_CASES = [(1500, 1100, 12), (1100, 1100, 12), (1100, 700, 0), (1497, 1100, 22)]
 
 
 @pytest.mark.parametrize("m,n,max_ctas", HALF_CASES)
@@ -479,10 +477,11 @@ def test_half_tile_tail(oracle_mod, m, n, max_ctas, tA, tB, out, beta):
     k = 520
     C = inputs.uniform_f16(m, n, 27).astype(np.float32 if out == "f32" else np.float16)
     opA, opB = inputs.uniform_f16(m, k, 25), inputs.uniform_f16(k, n, 26)
-    binding.set_config("tc2", block_n=512, max_ctas=max_ctas, stream_k=1)
+    binding.set_config("tc2", block_n=512, max_ctas=max_ctas, stream_k=1, half_tail=2)
     case = GpuCase(opA, opB, tA, tB, 1.0, beta, C=C, out=out, pad=(8, 16, 8))
     got, again = case.run_gpu(repeat=2)
     _expect_kernel(case, "tc2", 512)
+    assert case.stats["half_tail"] == 2, case.stats
     binding.set_config("tc2", block_n=256, max_ctas=max_ctas, stream_k=1)
     ref256 = GpuCase(opA, opB, tA, tB, 1.0, beta, C=C, out=out, pad=(8, 16, 8)).run_gpu()
     u = np.uint32 if out == "f32" else np.uint16
@@ -495,10 +494,25 @@ def test_half_tile_tail(oracle_mod, m, n, max_ctas, tA, tB, out, beta):
 
 def test_half_tile_tail_integer_exact(oracle_mod):
     from paper_conf_ipps_00020c20_b200 import binding
-    binding.set_config("tc2", block_n=512, max_ctas=12, stream_k=1)
+    binding.set_config("tc2", block_n=512, max_ctas=12, stream_k=1, half_tail=2)
     opA = inputs.integer_f16(1500, 1024, 3, -4, 4)
     opB = inputs.integer_f16(1024, 1100, 4, -4, 4)
     case = GpuCase(opA, opB, "T", "N", out="f32")
     got = case.view(case.run_gpu())
     _, r, _ = case.oracle(oracle_mod)
     assert np.array_equal(got.astype(np.float64), r)
+
+
+def test_half_tile_tail_regression_slow_epilogue(oracle_mod):
+    """The case that exposed a tmem_full parity alias (a half item as a CTA's third
+    work item, beta != 0, entirely outside N), run repeatedly."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("tc2", block_n=512, max_ctas=12, stream_k=1, half_tail=2)
+    m, n, k = 1100, 1100, 520
+    C = inputs.uniform_f16(m, n, 27).astype(np.float16)
+    case = GpuCase(inputs.uniform_f16(m, k, 25), inputs.uniform_f16(k, n, 26), "T", "N", 1.0, 1.0, C=C, out="f16")
+    outs = case.run_gpu(repeat=20)
+    assert case.stats["half_tail"] == 2
+    assert all(np.array_equal(o.view(np.uint16), outs[0].view(np.uint16)) for o in outs)
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, outs[0], r, ab)
