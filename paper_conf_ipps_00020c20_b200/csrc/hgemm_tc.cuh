@@ -338,7 +338,7 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
 // read it: empty[] counts MC arrivals, multicast by each pair's MMA leader.
 // Copy warp of the fused all-gather (AG = true; warp 2 + EPI_WARPS): pulls copy
 // units of op(A) rows from the peers' gather buffers (over NVLink: plain 16-B
-// loads from P2P-mapped memory) into the local one, 8 loads in flight per lane,
+// loads from P2P-mapped memory) into the local one, 16 loads in flight per lane,
 // and publishes each finished unit in its chunk's counter.  Units are taken from
 // a shared work index, so any subset of resident CTAs completes all of them.
 __device__ __forceinline__ void ag_copy_warp(const TcParams &p, uint32_t lane) {
@@ -364,7 +364,7 @@ __device__ __forceinline__ void ag_copy_warp(const TcParams &p, uint32_t lane) {
     const uint4 *src = static_cast<const uint4 *>(p.ag_peer[q]);
     uint4 *dst = static_cast<uint4 *>(p.ag_A);
     const int64_t total = (r1 - r0) * vpr;
-    constexpr int UNR = 8;
+    constexpr int UNR = 16;  // 8 KB in flight per copy warp (NVLink latency ~1-2 us)
     for (int64_t base = 0; base < total; base += 32 * UNR) {
       uint4 v[UNR];
       int64_t off[UNR];

@@ -76,7 +76,7 @@ def test_plan_random_cover():
 def test_plan_sharded_32768():
     world, m = 8, 32768
     cr = default_chunk_rows(m, world)
-    assert cr == 2048
+    assert cr == 4096
     rs = [slab_bounds(m, world, q, align=cr)[0] for q in range(world)] + [m]
     for rank in range(world):
         ops = _check_plan(m, rs, rank, cr)
