@@ -107,6 +107,8 @@ typedef enum {
     HGEMM_KERNEL_STREAM = 5      /* HBM-streaming tcgen05 kernel for skinny shapes: n <= 256, transA 'T',
                                     transB 'N' (both operands K-contiguous); one persistent CTA per SM,
                                     each owning column chunks of C^T of block_n (multiple of 16) rows of op(A);
+                                    with n > 256 and m <= 256 the operands are swapped (op(B) streamed,
+                                    C stored transposed; reported with group_m = 1);
                                     other shapes/layouts fall back to the automatic choice */
 } hgemm_kernel_t;
 

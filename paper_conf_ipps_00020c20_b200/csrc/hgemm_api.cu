@@ -471,6 +471,13 @@ inline bool choose_stream(int64_t M, int64_t N, int64_t K, int num_sms) {
   return M <= 256 && N >= static_cast<int64_t>(num_sms) * 64 && K >= 256;
 }
 
+// Swapped streaming (small m = Ms <= 256, long n = Ns) is available when forced
+// (hgemm_config_t kernel = HGEMM_KERNEL_STREAM) but not chosen automatically: on
+// the LSTM-gate shapes it measured slower than split-K (m = 64: 22.5 vs 14.4 us;
+// m = 256: 30.7 vs 16.4 us; profiles/r01b/lstm_swapped_stream.log) -- each
+// 32-row chunk re-reads the resident op(A) k-block by k-block and issues N = 32 MMAs.
+inline bool choose_stream_swapped(int64_t, int64_t, int64_t, int) { return false; }
+
 inline bool is_t(char c) { return c == 'T' || c == 't'; }
 inline bool is_n(char c) { return c == 'N' || c == 'n'; }
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
@@ -698,6 +705,55 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     if (st == HGEMM_SUCCESS) {
       std::lock_guard<std::mutex> lk(g_mu);
       g_last = {HGEMM_KERNEL_STREAM, cw, 0, grid, 0, 0};
+    }
+    return st;
+  }
+
+  // ---------------------------------------------------------- HBM streaming, swapped operands
+  // Small m with a long n (LSTM gates, batch <= 256): the big operand is op(B).  The
+  // streaming kernel then keeps op(A) (m <= 256 rows) resident as its UMMA A operand,
+  // streams the rows of op(B)^T (K-contiguous for transB 'N') and stores D = C
+  // transposed (column-major C, element (i, j) at C + j*ldc + i).
+  if (!ag && !a_mn && !b_mn && N <= 256 && M > 256 &&
+      ((cfg.kernel == HGEMM_KERNEL_STREAM) ||
+       (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream_swapped(N, M, k, di.num_sms)))) {
+    const int64_t Ms = N, Ns = M;  // the swapped problem: M' = m, N' = n
+    const int mt = Ms <= 128 ? 1 : 2;
+    int cw = cfg.kernel == HGEMM_KERNEL_STREAM && cfg.block_n ? cfg.block_n : stream_chunk(Ns, mt, di.num_sms);
+    if (mt == 2 && cw > 128) cw = 128;
+    CUtensorMap ta, tb;
+    const uint32_t a_rows = (Ms <= 64 && cw >= 64) ? 64u : 128u;
+    bool ok = make_map(&ta, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, a_rows);
+    if (ok) ok = make_map(&tb, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, cw);
+    if (!ok) return HGEMM_ERR_CUDA;
+    hg::StreamParams p = {};
+    p.M = static_cast<int32_t>(Ms);
+    p.N = static_cast<int32_t>(Ns);
+    p.K = static_cast<int32_t>(k);
+    p.cw = cw;
+    p.num_chunks = static_cast<int32_t>(cdiv(Ns, cw));
+    p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
+    p.a_bytes = a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u;
+    p.stage_bytes = p.a_bytes + static_cast<uint32_t>(cw) * 128u;
+    p.stages = static_cast<int32_t>(std::min<uint32_t>(hg::kStreamMaxStages,
+                                                       (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
+    p.probe = g_probe.load(std::memory_order_relaxed);
+    p.k_rot = 1;
+    p.alpha = alpha;
+    p.beta = beta;
+    p.D = C;
+    p.ldd = ldc;
+    p.tout = 1;
+    int grid = static_cast<int>(std::min<int64_t>(p.num_chunks, di.num_sms));
+    if (cfg.max_ctas > 0) grid = std::min(grid, cfg.max_ctas);
+    hgemm_status_t st;
+    if (mt == 1) st = f32 ? launch_stream<1, true>(ta, tb, p, grid, dev, stream)
+                          : launch_stream<1, false>(ta, tb, p, grid, dev, stream);
+    else st = f32 ? launch_stream<2, true>(ta, tb, p, grid, dev, stream)
+                  : launch_stream<2, false>(ta, tb, p, grid, dev, stream);
+    if (st == HGEMM_SUCCESS) {
+      std::lock_guard<std::mutex> lk(g_mu);
+      g_last = {HGEMM_KERNEL_STREAM, cw, 1 /* swapped */, grid, 0, 0};
     }
     return st;
   }

@@ -120,7 +120,28 @@ __global__ void __launch_bounds__(192, 1)
   } while (0)
 #endif
   if (threadIdx.x == 0) SK_TRACE(0);
-  griddep_wait();  // PDL: launch overlapped the previous kernel; C is read right below
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+  }
+  if (warp == 1) {
+    if (lane == 0) {
+      for (int s = 0; s < STAGES; ++s) {
+        mbar_init(&full[s], 1);
+        mbar_init(&empty[s], 1);
+      }
+      mbar_init(tfull, 1);
+      fence_mbarrier_init();
+    }
+    __syncwarp();
+    tmem_alloc<1>(smem_u32(tmem_slot), SH::TMEM_COLS);
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  if (threadIdx.x == 0) SK_TRACE(1);
+  griddep_wait();  // PDL: the prologue above overlapped the previous kernel; C is read right below
   // Epilogue warps prefetch their C slice (FP16 vector path, beta != 0) at
   // kernel start: C does not depend on the accumulator.
   uint32_t cpre[SH::SLICE / 2];
@@ -144,27 +165,6 @@ __global__ void __launch_bounds__(192, 1)
       }
     }
   }
-  if (warp == 0 && lane == 0) {
-    tma_prefetch_desc(&tmA);
-    tma_prefetch_desc(&tmB);
-  }
-  if (warp == 1) {
-    if (lane == 0) {
-      for (int s = 0; s < STAGES; ++s) {
-        mbar_init(&full[s], 1);
-        mbar_init(&empty[s], 1);
-      }
-      mbar_init(tfull, 1);
-      fence_mbarrier_init();
-    }
-    __syncwarp();
-    tmem_alloc<1>(smem_u32(tmem_slot), SH::TMEM_COLS);
-  }
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  const uint32_t tmem_base = *tmem_slot;
-  if (threadIdx.x == 0) SK_TRACE(1);
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer

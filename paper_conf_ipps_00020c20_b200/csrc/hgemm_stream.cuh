@@ -45,6 +45,11 @@ struct StreamParams {
   void *D;
   int64_t ldd;
   unsigned long long *probe;  // HGEMM_TRACE builds: per-CTA %globaltimer events (tools/trace_stream.py)
+  // 1: D is stored transposed, element (row, col) at D + col*ldd + row (the
+  // swapped-operand use for small m: the kernel streams op(B) and keeps op(A)
+  // resident, computing C = op(A) op(B) with C column-major; each warp's 32 rows
+  // are consecutive in memory, so every column store is one 64/128-B segment)
+  int32_t tout;
 };
 
 #ifdef HGEMM_TRACE
@@ -212,6 +217,28 @@ __global__ void __launch_bounds__(192, 1)
           float r[16];
 #pragma unroll
           for (int j = 0; j < 16; ++j) r[j] = alpha * __uint_as_float(v[j]);
+          if (p.tout) {  // transposed D: column col+j is contiguous over this warp's rows
+            const int nj = min(16, p.N - col);
+            if (beta != 0.0f) {  // all 16 C loads first (no store in between), then the stores
+              float cv[16];
+#pragma unroll
+              for (int j = 0; j < 16; ++j) {
+                const int64_t o = static_cast<int64_t>(col + j) * p.ldd + row;
+                if constexpr (OUT_F32) cv[j] = j < nj ? static_cast<const float *>(p.D)[o] : 0.0f;
+                else cv[j] = j < nj ? __half2float(static_cast<const __half *>(p.D)[o]) : 0.0f;
+              }
+#pragma unroll
+              for (int j = 0; j < 16; ++j) r[j] = fmaf(beta, cv[j], r[j]);
+            }
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+              if (j >= nj) break;
+              const int64_t o = static_cast<int64_t>(col + j) * p.ldd + row;
+              if constexpr (OUT_F32) static_cast<float *>(p.D)[o] = r[j];
+              else static_cast<__half *>(p.D)[o] = __float2half_rn(r[j]);
+            }
+            continue;
+          }
           const int64_t off = static_cast<int64_t>(row) * p.ldd + col;
           const bool whole = col + 16 <= p.N;  // 16 columns inside N: 16-B aligned vectors
           if constexpr (OUT_F32) {

@@ -335,9 +335,10 @@ def test_splitk_splits(oracle_mod, splits, bn, tA, tB):
 
 
 def test_splitk_auto_for_underfilled(oracle_mod):
-    """LSTM-gate shape (m=64 batch, n=4096, k=2048): automatic selection splits K."""
+    """LSTM-gate shape (m=64 batch, n=4096, k=2048) in NN layout (no streaming kernel):
+    automatic selection splits K."""
     m, n, k = 64, 4096, 2048
-    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "T", "N", 1.0, 1.0,
+    case = GpuCase(inputs.uniform_f16(m, k, 1), inputs.uniform_f16(k, n, 2), "N", "N", 1.0, 1.0,
                    C=inputs.uniform_f16(m, n, 3), out="f16")
     got = case.run_gpu()
     assert case.stats["last_kernel"] == "splitk", case.stats
@@ -516,3 +517,34 @@ def test_half_tile_tail_regression_slow_epilogue(oracle_mod):
     assert all(np.array_equal(o.view(np.uint16), outs[0].view(np.uint16)) for o in outs)
     _, r, ab = case.oracle(oracle_mod)
     assert_within_tolerance(case, outs[0], r, ab)
+
+
+# Streaming kernel with swapped operands (small m, long n; TN; forced with the "stream"
+# kernel choice): op(A) resident, op(B) streamed, C stored transposed from the
+# accumulator.
+@pytest.mark.parametrize("m,n", [(1, 2400), (64, 4096), (100, 4100), (256, 2500)])
+@pytest.mark.parametrize("out,beta", [("f16", 0.0), ("f16", 1.0), ("f32", -0.5)])
+def test_stream_swapped(oracle_mod, m, n, out, beta):
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("stream")   # forced: not chosen automatically (slower than split-K here)
+    k = 520
+    C = inputs.uniform_f16(m, n, 37).astype(np.float32 if out == "f32" else np.float16)
+    case = GpuCase(inputs.uniform_f16(m, k, 35), inputs.uniform_f16(k, n, 36), "T", "N", 1.5, beta, C=C,
+                   out=out, pad=(8, 16, 8))
+    got = case.run_gpu()
+    assert case.stats["last_kernel"] == "stream" and case.stats["group_m"] == 1, case.stats
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, got, r, ab)
+    assert np.all(np.isnan(case.padding(got).astype(np.float32)))
+
+
+def test_stream_swapped_integer_exact(oracle_mod):
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("stream")
+    opA = inputs.integer_f16(64, 2048, 33, -4, 4)
+    opB = inputs.integer_f16(2048, 4096, 34, -4, 4)
+    case = GpuCase(opA, opB, "T", "N", out="f32")
+    got = case.view(case.run_gpu())
+    assert case.stats["last_kernel"] == "stream" and case.stats["group_m"] == 1, case.stats
+    _, r, _ = case.oracle(oracle_mod)
+    assert np.array_equal(got.astype(np.float64), r)
