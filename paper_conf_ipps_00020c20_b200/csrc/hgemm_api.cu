@@ -45,6 +45,15 @@ std::atomic<int64_t> g_launches{0};
 std::atomic<unsigned long long *> g_probe{nullptr};
 // programmatic dependent launch of the tensor-core kernels (HGEMM_PDL=0 disables it: experiments)
 thread_local bool t_half_used = false;  // the last tile launch of this thread used the half-tile tail
+// experiment knobs, read once at load time (never per call)
+int env_int(const char *name, int dflt) {
+  const char *e = std::getenv(name);
+  return e ? std::atoi(e) : dflt;
+}
+const int g_env_stream_rot = env_int("HGEMM_STREAM_ROT", 1);  // streaming kernel k rotation
+const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pair kernel (-DHGEMM_ENABLE_MC)
+const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster groups along N
+const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hints
 const bool g_pdl = [] {
   const char *e = std::getenv("HGEMM_PDL");
   return !(e && e[0] == '0');
@@ -689,8 +698,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     p.stages = static_cast<int32_t>(std::min<uint32_t>(hg::kStreamMaxStages,
                                                        (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
     p.probe = g_probe.load(std::memory_order_relaxed);
-    p.k_rot = 1;
-    if (const char *e = std::getenv("HGEMM_STREAM_ROT")) p.k_rot = std::atoi(e);  // experiments
+    p.k_rot = g_env_stream_rot;
     p.alpha = alpha;
     p.beta = beta;
     p.D = C;
@@ -818,7 +826,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   int mc = 1;
 #ifdef HGEMM_ENABLE_MC
   if (cg == 2 && !ag) {
-    if (const char *e = std::getenv("HGEMM_MC")) mc = std::atoi(e) == 2 ? 2 : 1;  // experiments
+    mc = g_env_mc == 2 ? 2 : 1;  // experiments
   }
 #endif
 
@@ -844,14 +852,9 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
   p.group_m = cfg.group_m > 0 ? cfg.group_m : 16 / mc;  // measured best with 256x512 pair tiles (profiles/)
   p.group_m = std::max(1, std::min(p.group_m, p.num_m_tiles));
-  if (const char *e = std::getenv("HGEMM_GROUP_N")) {  // experiments: group along N instead
-    const int gn = std::atoi(e);
-    if (gn > 0) p.group_m = -std::max(1, std::min(gn, p.num_n_tiles));
-  }
-  {
-    const char *e = std::getenv("HGEMM_L2_HINT");
-    p.l2_hint = e ? std::atoi(e) : 0;
-  }
+  if (g_env_group_n > 0)  // experiments: group along N instead
+    p.group_m = -std::max(1, std::min(g_env_group_n, p.num_n_tiles));
+  p.l2_hint = g_env_l2_hint;
   if (ag) {
     p.ag_ctr = ag->ctr;
     for (int q = 0; q < ag->world; ++q) p.ag_peer[q] = ag->peers[q];
