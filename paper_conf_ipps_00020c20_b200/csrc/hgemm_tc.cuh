@@ -794,6 +794,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       int tm, tn, itile, isub;
       item_tile(p, wi.tile, itile, isub);
       tile_coords(itile, p, tm, tn);
+      WorkItem wnext;
+      const bool last_item = !get_item(p, cluster_id, num_clusters, i + 1, wnext);
       // half item: accumulator half 0 holds D columns tn*BN + isub*UMMA_N ..; half 1 is
       // only handed back (nh_act accumulator halves carry data)
       const bool half = (NH == 2 && MC == 1 && isub >= 0);
@@ -1003,6 +1005,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             }
           }
           if (warp == 2 && lane == 0) HG_TRACE(it, 10 + h);
+#ifdef HGEMM_TRACE
+          if (warp == 2 && lane == 0 && it == 0 && h == 0) HG_STAMP2(5);
+#endif
           tc_fence_before();
           __syncwarp();
           if (lane == 0) {
@@ -1011,11 +1016,29 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             else mbar_arrive_relaxed(&tempty[buf * NH + h]);
             if (warp == 2) HG_TRACE(it, 2 + h);
           }
+          // The last accumulator half of a CTA's last work item: every MMA has retired
+          // and no operand load is pending, so the smem ring is free -- stage every box
+          // in its own ring slot instead of waiting for the staging buffer to be read.
+          constexpr int RB = EPI_COLS_W / EPI_COLS;  // boxes per warp per accumulator half
+          static_assert(S::EPI_WARPS * RB * 4096u <= STAGES * STAGE_BYTES, "ring staging");
+          if (last_item && p.sk_units == 0 && hh == NH - 1) {
 #pragma unroll
-          for (int c = 0; c < EPI_COLS_W / EPI_COLS; ++c)
-            emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, stg, nstore,
-                                                     *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
-                                                     cbase + c0 + c * EPI_COLS, row, row_base, lane);
+            for (int c = 0; c < RB; ++c) {
+              uint32_t ns = 0;  // < EPI_BUFS: no buffer wait
+              emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, smem_u32(smem) + (ew * RB + c) * 4096u, ns,
+                                                       *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
+                                                       cbase + c0 + c * EPI_COLS, row, row_base, lane);
+            }
+          } else {
+#pragma unroll
+            for (int c = 0; c < RB; ++c)
+              emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, stg, nstore,
+                                                       *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
+                                                       cbase + c0 + c * EPI_COLS, row, row_base, lane);
+          }
+#ifdef HGEMM_TRACE
+          if (warp == 2 && lane == 0 && it == 0 && h == 0) HG_STAMP2(6);
+#endif
         }
         continue;
       }
@@ -1184,6 +1207,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
     // global writes complete with the grid (the next kernel's griddepcontrol.wait
     // or stream order sees them)
     if (lane == 0) bulk_wait_group_read<0>();
+#ifdef HGEMM_TRACE
+    if (warp == 2 && lane == 0) HG_STAMP2(7);
+#endif
   }
 
   // Reconverge each warp (the role code ran on one lane of warps 0/1) before the

@@ -50,7 +50,8 @@ for f, nm in names:
         print(f"  {nm:9s} n={len(xs):3d} min {min(xs) / 1e3:7.2f} med {statistics.median(xs) / 1e3:7.2f} "
               f"max {max(xs) / 1e3:7.2f} us")
 rows2 = [v[264 + 1280 + 8 * b: 264 + 1280 + 8 * b + 8] for b in range(160) if v[264 + 8 * b]]
-for f, nm in [(0, "prod_start"), (1, "item0"), (2, "empty0"), (3, "expect_tx"), (4, "tmaA0")]:
+for f, nm in [(0, "prod_start"), (1, "item0"), (2, "empty0"), (3, "expect_tx"), (4, "tmaA0"),
+              (5, "epi_tmem"), (6, "epi_stores"), (7, "epi_wait")]:
     xs = [r[f] - t0 for r in rows2 if r[f]]
     if xs:
         print(f"  {nm:10s} n={len(xs):3d} min {min(xs) / 1e3:7.2f} med {statistics.median(xs) / 1e3:7.2f} "
