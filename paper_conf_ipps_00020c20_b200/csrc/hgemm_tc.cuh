@@ -888,7 +888,18 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       if (c_tma) {
         // per staging box: TMEM -> registers, wait for its C box, alpha*acc + beta*C
         // in FP32 in place, TMA store; a half goes back to the MMA warp after its
-        // last box's TMEM read, a box after its store has read it takes the next C box
+        // last box's TMEM read, a box after its store has read it takes the next C box.
+        // A CTA's last work item with one accumulator half (NH == 1): the MMAs have
+        // retired, so the smem ring is free -- the remaining C boxes are all loaded
+        // at once into ring slots (skbar[ew][1]) instead of one after another.
+        const bool ring_c = (NH == 1) && (EPI_BUFS == 1) && last_item && p.sk_units == 0 && nbt > EPI_BUFS;
+        static_assert(NH != 1 || S::EPI_WARPS * NBT * 4096u <= STAGES * STAGE_BYTES, "ring staging of C");
+        auto ring_slot = [&](int j) { return smem_u32(smem) + (ew * NBT + j) * 4096u; };
+        if (ring_c && lane == 0) {
+          mbar_arrive_expect_tx(&skbar[ew * 2 + 1], static_cast<uint32_t>(nbt - EPI_BUFS) * 4096u);
+          for (int j = EPI_BUFS; j < nbt; ++j)
+            tma_load_2d(&tmD, ring_slot(j), smem_u32(&skbar[ew * 2 + 1]), box_col(j), row_base, 0);
+        }
 #pragma unroll 1
         for (int hh = 0; hh < NH; ++hh) {
           const int h = half_at(hh);
@@ -923,10 +934,17 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
                 if (warp == 2) HG_TRACE(it, 2 + h);
               }
             }
+            const bool in_ring = ring_c && j >= EPI_BUFS;
             const uint32_t b = (s0 + static_cast<uint32_t>(j)) % EPI_BUFS;
-            mbar_wait(&skbar[ew * 2 + b], sk_uses[b] & 1u);
-            ++sk_uses[b];
-            const uint32_t sbuf = stg + b * (32u * 128u);
+            uint32_t sbuf;
+            if (in_ring) {
+              mbar_wait(&skbar[ew * 2 + 1], 0u);  // single use per launch
+              sbuf = ring_slot(j);
+            } else {
+              mbar_wait(&skbar[ew * 2 + b], sk_uses[b] & 1u);
+              ++sk_uses[b];
+              sbuf = stg + b * (32u * 128u);
+            }
             const uint32_t rowaddr = sbuf + lane * 128u;
 #pragma unroll
             for (int q = 0; q < 8; ++q) {
@@ -954,7 +972,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             if (lane == 0) {
               tma_store_2d(&tmD, sbuf, cbase + colt, row_base);
               bulk_commit_group();
-              if (j + EPI_BUFS < nbt) {
+              if (!ring_c && j + EPI_BUFS < nbt) {
                 bulk_wait_group_read<0>();  // this box's store has read it: load the next C box
                 c_load(j + EPI_BUFS);
               }
