@@ -85,6 +85,15 @@ def test_baseline_configs(oracle_mod, name):
 
 
 @pytest.mark.slow
+@pytest.mark.parametrize("w,beta,out", [(7168, 0.0, "f16"), (6400, 1.0, "f16"), (7680, 0.0, "f32")])
+def test_half_tile_tail_full_size(oracle_mod, w, beta, out):
+    """Square sizes of the paper sweep where the automatic choice runs 512-wide tiles
+    with the half-tile tail: sampled entries, tile edges."""
+    got, stats = _check_sampled(oracle_mod, w, w, w, "T", "N", 1.0, beta, out, seed=300)
+    assert stats["last_kernel"] == "tc2" and stats["block_n"] == 512 and stats["half_tail"] == 2, stats
+
+
+@pytest.mark.slow
 def test_vs_cublas_full_matrix():
     """Whole-matrix cross-check against cuBLAS (torch.mm, FP32 accumulation forced)."""
     import torch
