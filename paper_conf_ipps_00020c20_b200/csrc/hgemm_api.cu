@@ -54,6 +54,7 @@ const int g_env_stream_rot = env_int("HGEMM_STREAM_ROT", 1);  // streaming kerne
 const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pair kernel (-DHGEMM_ENABLE_MC)
 const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster groups along N
 const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hints
+const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
 const bool g_pdl = [] {
   const char *e = std::getenv("HGEMM_PDL");
   return !(e && e[0] == '0');
@@ -855,6 +856,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   if (g_env_group_n > 0)  // experiments: group along N instead
     p.group_m = -std::max(1, std::min(g_env_group_n, p.num_n_tiles));
   p.l2_hint = g_env_l2_hint;
+  p.exp_flags = g_env_exp;
   if (ag) {
     p.ag_ctr = ag->ctr;
     for (int q = 0; q < ag->world; ++q) p.ag_peer[q] = ag->peers[q];

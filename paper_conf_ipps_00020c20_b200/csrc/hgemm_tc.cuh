@@ -83,6 +83,7 @@ struct TcParams {
   // 1, accumulator half 0 only), so a last wave of R <= units/2 tiles takes half
   // the time.  Work items are numbered over tiles + n_half virtual items.
   int32_t n_half;
+  int32_t exp_flags;  // experiments (HGEMM_EXP): 1 = no ring staging for the last item, 2 = no C-load hold-back
 };
 
 // One unit of work of a cluster: k-blocks [kb0, kb1) of cluster tile `tile`.
@@ -849,7 +850,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         tma_load_2d(&tmD, stg + b * (32u * 128u), smem_u32(&skbar[ew * 2 + b]), box_col(j), row_base, 0);
       };
       if (c_tma && lane == 0) {
-        if (it == 0) mbar_wait(cgo, 0);  // behind the first operand stages in the memory queues
+        if (it == 0 && !(p.exp_flags & 2)) mbar_wait(cgo, 0);  // behind the first operand stages in the memory queues
         bulk_wait_group_read<0>();  // earlier stores have read every staging box of this warp
 #pragma unroll
         for (int j = 0; j < NBT; ++j) {
@@ -892,7 +893,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         // A CTA's last work item with one accumulator half (NH == 1): the MMAs have
         // retired, so the smem ring is free -- the remaining C boxes are all loaded
         // at once into ring slots (skbar[ew][1]) instead of one after another.
-        const bool ring_c = (NH == 1) && (EPI_BUFS == 1) && last_item && p.sk_units == 0 && nbt > EPI_BUFS;
+        const bool ring_c = (NH == 1) && (EPI_BUFS == 1) && last_item && p.sk_units == 0 && nbt > EPI_BUFS &&
+                            !(p.exp_flags & 1);
         static_assert(NH != 1 || S::EPI_WARPS * NBT * 4096u <= STAGES * STAGE_BYTES, "ring staging of C");
         auto ring_slot = [&](int j) { return smem_u32(smem) + (ew * NBT + j) * 4096u; };
         if (ring_c && lane == 0) {
@@ -1039,7 +1041,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           // in its own ring slot instead of waiting for the staging buffer to be read.
           constexpr int RB = EPI_COLS_W / EPI_COLS;  // boxes per warp per accumulator half
           static_assert(S::EPI_WARPS * RB * 4096u <= STAGES * STAGE_BYTES, "ring staging");
-          if (last_item && p.sk_units == 0 && hh == NH - 1) {
+          if (last_item && p.sk_units == 0 && hh == NH - 1 && !(p.exp_flags & 1)) {
 #pragma unroll
             for (int c = 0; c < RB; ++c) {
               uint32_t ns = 0;  // < EPI_BUFS: no buffer wait
