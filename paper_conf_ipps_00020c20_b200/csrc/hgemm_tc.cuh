@@ -796,7 +796,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       item_tile(p, wi.tile, itile, isub);
       tile_coords(itile, p, tm, tn);
       WorkItem wnext;
-      const bool last_item = !get_item(p, cluster_id, num_clusters, i + 1, wnext);
+      const bool last_item = p.sk_units == 0 && !get_item(p, cluster_id, num_clusters, i + 1, wnext);
       // half item: accumulator half 0 holds D columns tn*BN + isub*UMMA_N ..; half 1 is
       // only handed back (nh_act accumulator halves carry data)
       const bool half = (NH == 2 && MC == 1 && isub >= 0);
