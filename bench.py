@@ -133,15 +133,19 @@ def dist_env():
     return world, rank, local
 
 
-def max_over_ranks(x, world):
+def max_over_ranks(x, world, op="max"):
     if world == 1:
         return x
     import torch
     import torch.distributed as dist
     dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
     t = torch.tensor([x], dtype=torch.float64, device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.MIN)
     return float(t.item())
+
+
+def min_over_ranks(x, world):
+    return max_over_ranks(x, world, op="min")
 
 
 # ------------------------------------------------------------------ reference arm (oracle)
@@ -209,14 +213,34 @@ def run_reference(args, world, rank):
             "scaling": "strong" if args.workload in inputs.STRONG_SCALING else "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
             "config": {"workload": args.workload, "m": m, "n": n, "k": k, "layout": tA + tB, "out": out},
-            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample,
+                             "host": host_info()},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
 
 
+def host_info():
+    """The host the oracle ran on: nproc, CPUs in this process's affinity mask, CPU model."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:  # pragma: no cover
+        pass
+    try:
+        aff = len(os.sched_getaffinity(0))
+    except AttributeError:  # pragma: no cover
+        aff = None
+    return {"nproc": os.cpu_count(), "affinity_cpus": aff, "cpu_model": model}
+
+
 def cpu_baseline(workload, budget_s=12.0):
-    """The oracle, as it stands, on the host cores over a bounded block of the workload."""
+    """The oracle, as it stands, on the host cores over a bounded block of the workload:
+    all cores (OpenMP over output columns; the reported value) and one thread."""
     import oracle
     from paper_conf_ipps_00020c20_b200 import inputs
     oracle.build()
@@ -224,8 +248,13 @@ def cpu_baseline(workload, budget_s=12.0):
     threads = oracle.max_threads()
     ms, ns = _oracle_sample_size(workload, threads, budget_s)
     dt = _time_oracle(workload, ms, ns, threads)
+    ms1, ns1 = _oracle_sample_size(workload, 1, budget_s / 2)
+    dt1 = _time_oracle(workload, ms1, ns1, 1)
     return {"value": 2.0 * ms * ns * k / dt / 1e12, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": f"{ms} x {ns} block of C with the full k = {k} of {workload} ({dt:.1f} s)"}
+            "sample": f"{ms} x {ns} block of C with the full k = {k} of {workload} ({dt:.1f} s)",
+            "single_thread": {"value": 2.0 * ms1 * ns1 * k / dt1 / 1e12, "unit": UNIT, "cores": 1,
+                              "sample": f"{ms1} x {ns1} block of C, full k ({dt1:.1f} s)"},
+            "host": host_info()}
 
 
 # ------------------------------------------------------------------ L2 flush
@@ -245,6 +274,113 @@ class L2Flush:
         import torch
         self.w.zero_()
         torch.sum(self.r, dim=0, out=self.sink)
+
+
+# ------------------------------------------------------------------ timing helpers
+def timed(fn, flush, warmup, steps, stream=None):
+    """W warm-up calls, then `steps` calls each bracketed by CUDA events on `stream`
+    (default: torch's current stream) with an L2 flush before each, outside the events."""
+    import torch
+    for _ in range(warmup):
+        flush()
+        fn()
+    torch.cuda.synchronize()
+    evs = []
+    for _ in range(steps):
+        flush()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        fn()
+        e1.record(stream)
+        evs.append((e0, e1))
+    torch.cuda.synchronize()
+    ts = [a.elapsed_time(b) for a, b in evs]
+    return {"mean": statistics.mean(ts), "median": statistics.median(ts), "min": min(ts), "max": max(ts),
+            "n": len(ts)}
+
+
+def device_operands(dev, m, n, k, tA, tB, beta, out, seed=1234, seed_b=5678):
+    """Seeded device operands in column-major storage (a stored R x C matrix is a (C, R)
+    row-major tensor): A, B, C and their leading dimensions (bench-only)."""
+    import torch
+    from paper_conf_ipps_00020c20_b200 import inputs
+    sa, sb = inputs.stored_shape(m, k, tA), inputs.stored_shape(k, n, tB)
+    g = torch.Generator(device=dev).manual_seed(seed)
+    A = (torch.rand(sa[1], sa[0], generator=g, device=dev) * 2 - 1).half()
+    gb = torch.Generator(device=dev).manual_seed(seed_b)
+    B = (torch.rand(sb[1], sb[0], generator=gb, device=dev) * 2 - 1).half()
+    C = torch.zeros(n, m, dtype=torch.float32 if out == "f32" else torch.float16, device=dev)
+    if beta != 0:
+        C.uniform_(-1, 1)
+    return A, max(1, sa[0]), B, max(1, sb[0]), C
+
+
+def cublas_fn(A, B, C, tA, tB, alpha, beta):
+    """cuBLAS (torch.mm / torch.addmm) on the same operands, layout and alpha/beta as
+    hgemm(A, B, C): FP32 accumulation (reduced-precision reduction off); beta != 0
+    reads and rewrites C in place."""
+    import torch
+    torch.backends.cuda.matmul.allow_fp16_reduced_precision_reduction = False
+    # A.shape == (cols, rows) of the stored A, so op(A) = A ('T') or A.t() ('N'); likewise
+    # op(B) = B.t() ('N') or B ('T').  Column-major C (m x n) is the row-major (n x m)
+    # tensor C^T = op(B)^T op(A)^T.
+    opA = A if tA in ("T", "t") else A.t()
+    opB = B.t() if tB in ("N", "n") else B
+    X, Y = opB.t(), opA.t()
+    f32 = C.dtype == torch.float32
+
+    def fn():
+        if beta != 0:
+            if not f32:
+                return torch.addmm(C, X, Y, beta=beta, alpha=alpha, out=C)
+            return torch.addmm(C, X, Y, out_dtype=torch.float32, beta=beta, alpha=alpha, out=C)
+        if not f32:
+            return torch.mm(X, Y, out=C) if alpha == 1 else torch.mm(X, Y, out=C).mul_(alpha)
+        r = torch.mm(X, Y, out_dtype=torch.float32)
+        return C.copy_(r) if alpha == 1 else C.copy_(r).mul_(alpha)
+    return fn
+
+
+# BASELINE.json configs reported beside the metric line, each with cuBLAS on the same
+# operands (north_star (5); SURVEY 8(d)): config 1 (launch-bound: wall time), config 2 in
+# the other layouts / FP32 out, config 3 (DL shapes, beta = 1), config 4 (HBM-bound).
+SIDE_CONFIGS = ["cfg1_256_NN_f32", "cfg2_8192_NN_f16", "cfg2_8192_NT_f16", "cfg2_8192_TN_f32",
+                "cfg3_bert_ffn1_4096", "cfg3_bert_ffn1_16384", "cfg3_bert_ffn2_4096",
+                "cfg3_lstm_b64", "cfg3_lstm_b256", "cfg3_lstm_b1024",
+                "cfg4_skinny_n64", "cfg4_skinny_n128", "cfg4_skinny_n256"]
+
+
+def side_config(name, dev, flush, peaks, warmup, steps, compute=None):
+    """One BJ config: ours (automatic kernel choice, or hgemm_ex with `compute`) and cuBLAS,
+    device-resident inputs, L2 flushed between launches, mean of `steps` event-timed launches."""
+    from paper_conf_ipps_00020c20_b200 import binding, inputs
+    m, n, k, tA, tB, alpha, beta, out = inputs.WORKLOADS[name]
+    A, lda, B, ldb, C = device_operands(dev, m, n, k, tA, tB, beta, out, seed=99, seed_b=98)
+    if compute is None:
+        def ours():
+            binding.hgemm(m, n, k, alpha, A, lda, B, ldb, beta, C, m, tA, tB, out)
+    else:
+        def ours():
+            binding.hgemm_ex(m, n, k, alpha, A, lda, B, ldb, beta, C, m, tA, tB, out, compute=compute)
+    t_ours = timed(ours, flush, warmup, steps)
+    st = binding.get_stats()
+    t_cub = timed(cublas_fn(A, B, C, tA, tB, alpha, beta), flush, warmup, steps)
+    flops = 2.0 * m * n * k
+    esz = 4 if out == "f32" else 2
+    r = roofline_entry(m, n, k, beta, esz, t_ours["mean"], peaks, None)
+    rec = {"shape": [m, n, k], "layout": tA + tB, "alpha": alpha, "beta": beta, "out": out,
+           "ours_ms": t_ours["mean"], "ours_ms_median": t_ours["median"],
+           "ours_TFLOP/s": flops / (t_ours["mean"] * 1e-3) / 1e12,
+           "cublas_ms": t_cub["mean"], "cublas_TFLOP/s": flops / (t_cub["mean"] * 1e-3) / 1e12,
+           "ours_over_cublas": t_cub["mean"] / t_ours["mean"],
+           "bound": r["bound"], "achieved": r["achieved"], "unit": r["unit"], "frac": r["frac"],
+           "kernel": f"{st['last_kernel']}/{st['block_n']}" + (f" split {st['splits']}" if st["splits"] else ""),
+           "steps": steps}
+    if compute is not None:
+        rec["compute"] = compute
+    if name.startswith("cfg1"):
+        rec["note"] = "launch-latency bound (34 MFLOP): wall time per call is the figure of merit"
+    return rec
 
 
 # ------------------------------------------------------------------ roofline
@@ -275,40 +411,142 @@ def roofline_entry(m, n, k, beta, esz, ms, peaks, traffic):
                            f"(intensity {flops / byts:.0f} FLOP/B, ridge {ridge:.0f})"}
 
 
-def skinny_roofline(dev, flush, peaks, reps=20):
-    """BJ configs[3]: M=16384, N in {64,128,256}, K=4096 (TN, FP16 out), device-resident,
-    L2 flushed between launches; achieved GB/s of the algorithmic bytes vs the HBM peak."""
+# ------------------------------------------------------------------ config 5: 32768^3, N-sharded (strong)
+def strong_32768(args, world, rank, dev, flush, steps=5, warmup=2):
+    """BASELINE.json configs[4]: the GLOBAL 32768^3 TN FP16-out problem with the columns of
+    B and C split over the ranks (rank g: 32768 x 32768/G x 32768), A replicated.  Reports
+    t_gemm (max over ranks of the mean of `steps` event-timed launches), and for N > 1 the
+    exchange of A three ways (NCCL broadcast alone, broadcast then GEMM, broadcast
+    pipelined in row panels, all-gather fused into the GEMM kernel), each guarded so that a
+    failing leg records its error instead of losing the line.  Rank 0 also times the whole
+    problem alone (t1) so the record carries t1 / (N * t_gemm)."""
     import torch
-    from paper_conf_ipps_00020c20_b200 import binding, inputs
-    out = {}
-    for name in ("cfg4_skinny_n64", "cfg4_skinny_n128", "cfg4_skinny_n256"):
-        m, n, k, tA, tB, alpha, beta, o = inputs.WORKLOADS[name]
-        g = torch.Generator(device=dev).manual_seed(99)
-        sa, sb = inputs.stored_shape(m, k, tA), inputs.stored_shape(k, n, tB)
-        A = (torch.rand(sa[1], sa[0], generator=g, device=dev) * 2 - 1).half()
-        B = (torch.rand(sb[1], sb[0], generator=g, device=dev) * 2 - 1).half()
-        C = torch.empty(n, m, dtype=torch.float16, device=dev)
+    from paper_conf_ipps_00020c20_b200 import binding
+    from paper_conf_ipps_00020c20_b200.sharded import broadcast_A, hgemm_sharded, slab_bounds
+    m = n = k = 32768
+    n0, n1 = slab_bounds(n, world, rank)
+    ns = n1 - n0
+    A, lda, Bs, ldb, C = device_operands(dev, m, ns, k, "T", "N", 0.0, "f16", seed=4321, seed_b=8765 + rank)
+    stream = torch.cuda.current_stream()
+    rec = {"global_shape": [m, n, k], "layout": "TN", "out": "f16", "n_per_rank": ns, "world": world,
+           "steps": steps, "what": "per-rank hgemm on its N-slab; A replicated (reported separately)"}
 
-        def call():
-            binding.hgemm(m, n, k, alpha, A, sa[0], B, sb[0], beta, C, m, tA, tB, o)
-        for _ in range(3):
-            call()
-        ts = []
-        for _ in range(reps):
-            flush()
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            call()
-            e1.record()
-            ts.append((e0, e1))
-        torch.cuda.synchronize()
-        ms = statistics.mean(a.elapsed_time(b) for a, b in ts)
-        r = roofline_entry(m, n, k, beta, 2, ms, peaks, None)
-        st = binding.get_stats()
-        out[name] = {"ms": ms, "bound": r["bound"], "achieved": r["achieved"], "unit": r["unit"],
-                     "frac": r["frac"], "TFLOP/s": 2.0 * m * n * k / (ms * 1e-3) / 1e12,
-                     "kernel": f"{st['last_kernel']}/{st['block_n']}" + (f" split {st['splits']}" if st['splits'] else "")}
-    return out
+    def gemm():
+        binding.hgemm(m, ns, k, 1.0, A, lda, Bs, ldb, 0.0, C, m, "T", "N", "f16")
+    if world > 1:
+        torch.distributed.barrier()
+    t = timed(gemm, flush, warmup, steps, stream)
+    t_gemm = max_over_ranks(t["mean"], world)
+    rec["t_gemm_ms"] = t_gemm
+    rec["t_gemm_ms_rank_spread"] = [min_over_ranks(t["mean"], world), t_gemm]
+    rec["TFLOP/s_aggregate"] = 2.0 * m * n * k / (t_gemm * 1e-3) / 1e12
+    st = binding.get_stats()
+    rec["kernel"] = f"{st['last_kernel']}/{st['block_n']}"
+    if rank == 0 and not args.no_cublas:
+        try:
+            tc = timed(cublas_fn(A, Bs, C, "T", "N", 1.0, 0.0), flush, warmup, steps, stream)
+            rec["cublas_slab_ms"] = tc["mean"]
+            rec["cublas_slab_TFLOP/s"] = 2.0 * m * ns * k / (tc["mean"] * 1e-3) / 1e12
+        except Exception as e:  # pragma: no cover
+            rec["cublas_error"] = f"{type(e).__name__}: {e}"
+    if world > 1:
+        # t1: the whole problem on rank 0 alone (same kernel path), for t1 / (N * t_gemm)
+        t1 = None
+        if rank == 0:
+            try:
+                del C
+                B1 = torch.empty(n, k, dtype=torch.float16, device=dev).uniform_(-1, 1)
+                C1 = torch.empty(n, m, dtype=torch.float16, device=dev)
+                t1 = timed(lambda: binding.hgemm(m, n, k, 1.0, A, lda, B1, k, 0.0, C1, m, "T", "N", "f16"),
+                           flush, 1, 3, stream)["mean"]
+                del B1, C1
+                C = torch.empty(ns, m, dtype=torch.float16, device=dev)
+            except Exception as e:  # pragma: no cover
+                rec["t1_error"] = f"{type(e).__name__}: {e}"
+                C = torch.empty(ns, m, dtype=torch.float16, device=dev)
+        else:
+            pass
+        torch.distributed.barrier()
+        if rank == 0 and t1:
+            rec["t1_ms"] = t1
+            rec["efficiency_t1_over_N_tgemm"] = t1 / (world * t_gemm)
+        rec.update(exchange_legs(args, world, rank, m, n, k, A, lda, Bs, ldb, C, "T", "N", "f16", stream))
+    return rec
+
+
+def exchange_legs(args, world, rank, m, n_glob, k, A, lda, Bs, ldb, C, tA, tB, out, stream, reps=3):
+    """The replication of A for the N-slab sharded GEMM, timed three ways (north_star (3):
+    the exchange is reported separately from the GEMM): NCCL broadcast alone, broadcast
+    then GEMM, broadcast pipelined in row panels of op(A), and the all-gather fused into
+    the GEMM kernel (hgemm_allgather_a).  Device time, mean of `reps`, max over ranks.
+    Every leg is guarded: an error is recorded in place of its number."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_00020c20_b200.sharded import broadcast_A, hgemm_sharded, hgemm_sharded_overlapped
+    res = {}
+
+    def leg(name, fn, pre=None):
+        try:
+            fn()
+            torch.cuda.synchronize()
+            ts = []
+            for _ in range(reps):
+                if pre is not None:
+                    pre()
+                torch.cuda.synchronize()
+                dist.barrier()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                fn()
+                e1.record(stream)
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            res[name] = max_over_ranks(statistics.mean(ts), world)
+            res[name + "_spread"] = [min(ts), max(ts)]
+        except Exception as e:  # pragma: no cover
+            res[name] = None
+            res[name + "_error"] = f"{type(e).__name__}: {e}"[:300]
+            try:
+                torch.cuda.synchronize()
+            except Exception:
+                pass
+    res["a_bytes"] = A.numel() * 2
+    leg("ms_bcast", lambda: broadcast_A(A, src=0))
+    if res.get("ms_bcast"):
+        res["bcast_GB_s"] = A.numel() * 2 / (res["ms_bcast"] * 1e-3) / 1e9
+    res["bcast_backend"] = dist.get_backend()
+    leg("ms_bcast_then_gemm", lambda: hgemm_sharded(m, n_glob, k, 1.0, A, lda, Bs, ldb, 0.0, C, m, tA, tB, out,
+                                                    broadcast=True, local_slabs=True, stream=stream.cuda_stream))
+    if tA in ("T", "t"):
+        leg("ms_bcast_gemm_pipelined",
+            lambda: hgemm_sharded_overlapped(m, n_glob, k, 1.0, A, lda, Bs, ldb, 0.0, C, m, tA, tB, out,
+                                             panels=args.panels, local_slabs=True, stream=stream.cuda_stream))
+        res["pipeline_panels"] = args.panels
+        ag = None
+        try:
+            from paper_conf_ipps_00020c20_b200.sharded import FusedAllGatherA
+            ag = FusedAllGatherA(m, k, lda=lda)
+            r0, r1 = ag.own_rows
+            ag.own_view().copy_(A[r0:r1, :k])
+            torch.cuda.synchronize()
+            dist.barrier()
+            n_rank = C.shape[0]
+            leg("ms_allgather_gemm_fused",
+                lambda: ag(n_rank, 1.0, Bs, ldb, 0.0, C, m, tB, out, stream=stream.cuda_stream))
+            res["allgather_fused_chunk_rows"] = ag.chunk_rows
+            res["allgather_fused_gather_ok"] = bool(torch.equal(ag.A[:, :k], A[:, :k]))
+        except Exception as e:  # pragma: no cover
+            res["ms_allgather_gemm_fused"] = None
+            res["ms_allgather_gemm_fused_error"] = f"{type(e).__name__}: {e}"[:300]
+        finally:
+            try:
+                torch.cuda.synchronize()
+                dist.barrier()
+                if ag is not None:
+                    ag.close()
+            except Exception:
+                pass
+    return res
 
 
 # ------------------------------------------------------------------ fused all-gather, one GPU
@@ -363,7 +601,7 @@ def ag_virtual(args, m, n, k, alpha, beta, tB, out, flush):
 def run_ours(args, world, rank, local):
     import torch
     from paper_conf_ipps_00020c20_b200 import binding, inputs
-    from paper_conf_ipps_00020c20_b200.sharded import broadcast_A, hgemm_sharded, slab_bounds
+    from paper_conf_ipps_00020c20_b200.sharded import hgemm_sharded, slab_bounds
     # HGEMM_DIST_BACKEND=gloo lets several ranks share one GPU to exercise the N > 1
     # code path where only one GPU is available (no performance meaning).
     backend = os.environ.get("HGEMM_DIST_BACKEND", "nccl")
@@ -391,91 +629,19 @@ def run_ours(args, world, rank, local):
     n_rank = n1 - n0
     out_t = torch.float32 if out == "f32" else torch.float16
     esz = 4 if out == "f32" else 2
-    sa = inputs.stored_shape(m, k, tA)
-    sb_rank = inputs.stored_shape(k, n_rank, tB)
-    # device inputs, seeded on the device (bench-only large configs).
-    # Column-major storage: a stored R x C matrix is a (C, R) row-major tensor.
-    g = torch.Generator(device=dev).manual_seed(1234)
-    A = (torch.rand(sa[1], sa[0], generator=g, device=dev) * 2 - 1).half()
-    gb = torch.Generator(device=dev).manual_seed(5678 + rank)
-    Bs = (torch.rand(sb_rank[1], sb_rank[0], generator=gb, device=dev) * 2 - 1).half()   # this rank's slab
-    C = torch.zeros(n_rank, m, dtype=out_t, device=dev)                                   # this rank's slab
-    if beta != 0:
-        C.uniform_(-1, 1)
-    lda, ldb = sa[0], sb_rank[0]
+    # device inputs, seeded on the device (bench-only large configs);
+    # A is the replicated operand, Bs / C this rank's slabs
+    A, lda, Bs, ldb, C = device_operands(dev, m, n_rank, k, tA, tB, beta, out, seed=1234, seed_b=5678 + rank)
     flush = L2Flush(dev)
     stream = torch.cuda.current_stream()
-
-    # the sharded path's one collective: replicate A (rank 0's copy) over NCCL, timed separately
-    coll = None
-    if world > 1:
-        import torch.distributed as dist
-        for _ in range(2):
-            broadcast_A(A, src=0)
-        torch.cuda.synchronize()
-        dist.barrier()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        broadcast_A(A, src=0)
-        e1.record()
-        torch.cuda.synchronize()
-        bms = max_over_ranks(e0.elapsed_time(e1), world)
-        coll = {"op": f"broadcast(A) over {dist.get_backend()} (torch.distributed)", "bytes": A.numel() * 2, "ms": bms,
-                "GB_s": A.numel() * 2 / (bms * 1e-3) / 1e9,
-                "note": "reported separately from the GEMM (north_star (3)); not inside value"}
-        # broadcast + GEMM as one step: serial, and pipelined in row panels of op(A) (NEXT-2)
-        if tA in ("T", "t"):
-            from paper_conf_ipps_00020c20_b200.sharded import hgemm_sharded_overlapped
-
-            def serial():
-                hgemm_sharded(m, n_glob, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out,
-                              broadcast=True, local_slabs=True, stream=stream.cuda_stream)
-
-            def overlapped():
-                hgemm_sharded_overlapped(m, n_glob, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out,
-                                         panels=args.panels, local_slabs=True, stream=stream.cuda_stream)
-            for name, fn in (("ms_bcast_then_gemm", serial), ("ms_bcast_gemm_pipelined", overlapped)):
-                fn()
-                torch.cuda.synchronize()
-                dist.barrier()
-                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                e0.record()
-                fn()
-                e1.record()
-                torch.cuda.synchronize()
-                coll[name] = max_over_ranks(e0.elapsed_time(e1), world)
-            coll["pipeline_panels"] = args.panels
-            # the all-gather fused with the GEMM (hgemm_allgather_a): A row-sharded over the
-            # ranks, peers' rows pulled over NVLink by the copy engines chunk by chunk while
-            # the persistent kernel consumes each chunk once its flag is raised
-            from paper_conf_ipps_00020c20_b200.sharded import FusedAllGatherA
-            ag = FusedAllGatherA(m, k, lda=lda)
-            r0, r1 = ag.own_rows
-            ag.own_view().copy_(A[r0:r1, :k])
-
-            def fused():
-                ag(n_rank, alpha, Bs, ldb, beta, C, m, tB, out, stream=stream.cuda_stream)
-            tf = []
-            for it in range(3):
-                torch.cuda.synchronize()
-                dist.barrier()                       # peers' rows are complete and no longer being read
-                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                e0.record(stream)
-                fused()
-                e1.record(stream)
-                torch.cuda.synchronize()
-                if it:
-                    tf.append(e0.elapsed_time(e1))
-            coll["ms_allgather_gemm_fused"] = max_over_ranks(statistics.mean(tf), world)
-            coll["allgather_fused_chunk_rows"] = ag.chunk_rows
-            coll["allgather_fused_gather_ok"] = bool(torch.equal(ag.A[:, :k], A[:, :k]))
-            torch.cuda.synchronize()
-            dist.barrier()
-            ag.close()
+    compute = args.compute
 
     def step():
-        hgemm_sharded(m, n_glob, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out,
-                      broadcast=False, local_slabs=True, stream=stream.cuda_stream)
+        if compute == "f16":
+            binding.hgemm_ex(m, n_rank, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out, compute="f16")
+        else:
+            hgemm_sharded(m, n_glob, k, alpha, A, lda, Bs, ldb, beta, C, m, tA, tB, out,
+                          broadcast=False, local_slabs=True, stream=stream.cuda_stream)
 
     for _ in range(args.warmup):
         flush()
@@ -504,7 +670,7 @@ def run_ours(args, world, rank, local):
     torch.cuda.synchronize()
     clk = clocks.stop()
     pv = probe.view(-1, 4).cpu().tolist()
-    ghz = [(c1 - c0) / (n1 - n0) for c0, n0, c1, n1 in pv if n1 > n0]
+    ghz = [(c1 - c0) / (n1_ - n0_) for c0, n0_, c1, n1_ in pv if n1_ > n0_]
     if ghz:
         clk["sm_mhz_in_kernel_median"] = 1000.0 * statistics.median(ghz)
         clk["sm_mhz_in_kernel_min"] = 1000.0 * min(ghz)
@@ -517,64 +683,35 @@ def run_ours(args, world, rank, local):
     flops_total = 2.0 * m * n_glob * k
     value = flops_total / (ms * 1e-3) / 1e12
     peaks = load_peaks()
-    achieved = flops_rank / (ms_local * 1e-3) / 1e12
     stats = binding.get_stats()
+    if stats["last_kernel"] == "tc2" and compute == "f16":
+        stats["compute"] = "f16 accumulate (hgemm_ex)"
 
     # cuBLAS on the same box, same tensors and layout (reference point, north_star (5)),
-    # right after our timed region so that both see the same power-cap state (the
-    # PCIe-bound e2e leg below lets the GPU cool down)
+    # right after our timed region so that both see the same power-cap state
     cublas = None
     if not args.no_cublas and rank == 0:
         try:
-            torch.backends.cuda.matmul.allow_fp16_reduced_precision_reduction = False
-            # Storage tensors are the transposes of the column-major matrices:
-            # A.shape == (cols, rows) of the stored A, so op(A) = A ('T') or A.t() ('N');
-            # likewise op(B) = Bs.t() ('N') or Bs ('T').  Column-major C (m x n) is the
-            # row-major (n x m) tensor C^T = op(B)^T op(A)^T.
-            opA = A if tA in ("T", "t") else A.t()
-            opB = Bs.t() if tB in ("N", "n") else Bs
-            X, Y = opB.t(), opA.t()
-
-            # same alpha/beta semantics: beta != 0 reads and rewrites C in place (addmm)
-            Cc = C.clone() if beta != 0 else None
-
-            def cub():
-                if beta != 0:
-                    if out_t == torch.float16:
-                        return torch.addmm(Cc, X, Y, beta=beta, alpha=alpha, out=Cc)
-                    return torch.addmm(Cc, X, Y, out_dtype=torch.float32, beta=beta, alpha=alpha, out=Cc)
-                if out_t == torch.float16:
-                    return torch.mm(X, Y) if alpha == 1 else torch.mm(X, Y).mul_(alpha)
-                return torch.mm(X, Y, out_dtype=torch.float32)
-            ref_c = cub()
-            # same protocol as our timed region (W warm-up steps, then K flushed steps):
-            # under the 1 kW power cap the SM clock falls during a long run, so a shorter
-            # cuBLAS run would be timed at a higher clock than ours
-            for _ in range(args.warmup):
-                flush()
-                cub()
-            torch.cuda.synchronize()
-            ts = []
-            for _ in range(args.steps):
-                flush()
-                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                e0.record()
-                cub()
-                e1.record()
-                ts.append((e0, e1))
-            torch.cuda.synchronize()
-            # agreement with our C (both FP32-accumulated; loose sanity bound only)
-            diff = (ref_c.float() - C.float()).abs().max().item() if beta == 0 else None
-            cms = statistics.mean(a.elapsed_time(b) for a, b in ts)
-            cublas = {"value": flops_rank / (cms * 1e-3) / 1e12, "unit": UNIT, "ms": cms, "max_abs_diff_vs_ours": diff,
+            Cc = C.clone()
+            tc = timed(cublas_fn(A, Bs, Cc, tA, tB, alpha, beta), flush, args.warmup, args.steps, stream)
+            diff = (Cc.float() - C.float()).abs().max().item() if beta == 0 else None
+            cublas = {"value": flops_rank / (tc["mean"] * 1e-3) / 1e12, "unit": UNIT, "ms": tc["mean"],
+                      "ms_median": tc["median"], "max_abs_diff_vs_ours": diff,
                       "what": ("torch.addmm(C, ..., beta, alpha, out=C)" if beta != 0 else "torch.mm") +
-                              " (cuBLAS), same operands, layout and alpha/beta, fp16 reduced-precision reduction off"}
+                              " (cuBLAS), same operands, layout and alpha/beta, fp16 reduced-precision reduction off,"
+                              " same W warm-up and K flushed steps as ours"}
+            del Cc
         except Exception as e:  # pragma: no cover
             cublas = {"error": f"{type(e).__name__}: {e}"}
 
+    # the exchange of A for the default (weak-scaling) workload, reported separately
+    coll = None
+    if world > 1 and not args.no_exchange:
+        coll = exchange_legs(args, world, rank, m, n_glob, k, A, lda, Bs, ldb, C, tA, tB, out, stream)
+
     # e2e through the public C-ABI host-buffer call (hgemm_host): every step copies this
     # step's A and B from pinned host memory, runs the GEMM and copies C back, all
-    # inside the timed region (the library pipelines column panels on its own streams)
+    # inside the timed region (the library pipelines panels on its own streams)
     e2e = None
     if not args.no_e2e:
         hA = A.cpu().pin_memory()
@@ -599,11 +736,32 @@ def run_ours(args, world, rank, local):
                "h2d_bytes_per_step": (A.numel() + Bs.numel()) * 2 * world + (C.numel() * esz * world if beta else 0),
                "d2h_bytes_per_step": C.numel() * esz * world, "ms_per_step": ems,
                "api": "hgemm_host (C ABI, pinned host buffers, panelled H2D/GEMM/D2H pipeline)"}
+        del hA, hB, hC, ws
 
-    # the HBM-bound skinny configs (BJ configs[3]) against the HBM roofline (north_star (5))
+    # config 5 (32768^3 N-sharded, strong scaling) at every N; guarded
+    strong_rec = None
+    if not args.no_strong and args.workload != "cfg5_sharded_32768":
+        try:
+            strong_rec = strong_32768(args, world, rank, dev, flush)
+        except Exception as e:  # pragma: no cover
+            strong_rec = {"error": f"{type(e).__name__}: {e}"[:300]}
+        torch.cuda.empty_cache()
+
+    # every other BJ config with cuBLAS beside it, and the FP16-accumulate compute type (rank 0, N = 1)
     side = None
     if rank == 0 and world == 1 and not args.no_side and args.workload == "cfg2_8192_TN_f16":
-        side = skinny_roofline(dev, flush, peaks)
+        side = {}
+        sst = max(5, min(args.steps, 30))
+        for name in SIDE_CONFIGS:
+            try:
+                side[name] = side_config(name, dev, flush, peaks, 5, sst)
+            except Exception as e:  # pragma: no cover
+                side[name] = {"error": f"{type(e).__name__}: {e}"[:300]}
+        try:
+            side["cfg2_8192_TN_f16_acc16"] = side_config("cfg2_8192_TN_f16", dev, flush, peaks, 5, sst, compute="f16")
+        except Exception as e:  # pragma: no cover
+            side["cfg2_8192_TN_f16_acc16"] = {"error": f"{type(e).__name__}: {e}"[:300]}
+        torch.cuda.empty_cache()
 
     agv = None
     if rank == 0 and world == 1 and args.ag_virtual > 0 and tA in ("T", "t"):
@@ -617,11 +775,16 @@ def run_ours(args, world, rank, local):
         peak = peaks["tflops_burst"]
         traffic = load_traffic(args.workload)
         roof = roofline_entry(m, n_rank, k, beta, esz, ms_local, peaks, traffic)
+        if roof["bound"] == "tensor" and peaks.get("tflops_sustained"):
+            roof["frac_vs_sustained_peak"] = roof["achieved"] / peaks["tflops_sustained"]
+            roof["sustained_peak"] = peaks["tflops_sustained"]
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "strong" if strong else "weak",
-            "vs_baseline": None, "dtype": "f16xf16->f32 (" + out + " out)", "data": "synthetic",
+            "vs_baseline": None,
+            "dtype": "f16xf16->" + ("f16 accumulate" if compute == "f16" else "f32") + " (" + out + " out)",
+            "data": "synthetic",
             "config": {"workload": args.workload, "m": m, "n": n_glob, "k": k, "n_per_gpu_rank0": n_rank,
                        "layout": tA + tB, "alpha": alpha, "beta": beta, "out": out,
                        "kernel": stats, "l2": "flushed between steps, outside the events: 256 MiB write, then a 256 MiB read so the write's dirty lines are written back before the timed launch",
@@ -634,7 +797,9 @@ def run_ours(args, world, rank, local):
             "cublas": cublas,
             "cpu_baseline": cpu,
             "collective": coll,
-            "hbm_bound_configs": side,
+            "strong_32768": strong_rec,
+            "bj_configs": side,
+            "hbm_bound_configs": ({kk: v for kk, v in side.items() if v.get("bound") == "hbm"} if side else None),
             "allgather_fused_virtual": agv,
             "step_ms": {"min": min(step_ms), "median": statistics.median(step_ms), "max": max(step_ms)},
         }
@@ -667,7 +832,11 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cublas", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--no-side", action="store_true", help="skip the skinny-shape HBM roofline report")
+    ap.add_argument("--no-side", action="store_true", help="skip the other BJ configs (bj_configs)")
+    ap.add_argument("--no-strong", action="store_true", help="skip the 32768^3 N-sharded record (strong_32768)")
+    ap.add_argument("--no-exchange", action="store_true", help="N > 1: skip the exchange-of-A legs")
+    ap.add_argument("--compute", default="f32", choices=["f32", "f16"],
+                    help="accumulation type of the timed step (f16: hgemm_ex FP16 accumulate, FP16 out)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     world, rank, local = dist_env()

@@ -39,7 +39,8 @@
  * Fast path (tcgen05 tensor cores + TMA): A and B 16-byte aligned, lda and
  * ldb multiples of 8 elements, C 16-byte aligned and ldc*sizeof(out) a
  * multiple of 16 bytes.  Anything else runs a slower CUDA-core kernel with
- * the same semantics (never an error).  All indexing is 64-bit.
+ * the same semantics (never an error; n > 65535*64 runs as several launches
+ * over column ranges).  All indexing is 64-bit.
  *
  * Thread safety: hgemm() is reentrant; per-device properties are cached.
  * hgemm_set_config() is process-global and meant for tests and benchmarks.
@@ -72,6 +73,33 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k,
                      char transA, char transB, hgemm_dtype_t out_dtype,
                      cudaStream_t stream);
 
+/* Accumulation type of hgemm_ex (like cublasGemmEx's computeType).
+ *   HGEMM_COMPUTE_F32: products accumulated in FP32 (what hgemm() does; BASELINE.json
+ *                      north_star (1)).
+ *   HGEMM_COMPUTE_F16: products accumulated in FP16 on the tensor cores
+ *                      (tcgen05.mma kind::f16 with an FP16 accumulator, c_format = F16):
+ *                      the paper's own precision mode, HMMA.1688.F16 (SIV-A;
+ *                      its register budget only fits FP16 accumulators, SVI-A.3).
+ *                      The epilogue still computes alpha*acc + beta*c in FP32 and rounds
+ *                      once to FP16.  Requires out_dtype == HGEMM_OUT_F16.  Accuracy:
+ *                      the FP16 accumulator loses the low bits of partial sums above 2048
+ *                      (11-bit significand); integer sums stay exact only while every
+ *                      partial sum is an integer of magnitude <= 2048. */
+typedef enum { HGEMM_COMPUTE_F32 = 0, HGEMM_COMPUTE_F16 = 1 } hgemm_compute_t;
+
+/* hgemm() with an explicit accumulation type; same arguments, layout, ownership,
+ * asynchrony, quick returns and fallback rules as hgemm().  Errors as hgemm(),
+ * plus HGEMM_ERR_INVALID_VALUE for an unknown compute type or HGEMM_COMPUTE_F16
+ * with out_dtype != HGEMM_OUT_F16.  The fast path uses the CTA-pair tile kernels
+ * (whole tiles, no stream-K / split-K / streaming kernels); the CUDA-core
+ * fallback rounds its accumulator to FP16 after every product. */
+hgemm_status_t hgemm_ex(int64_t m, int64_t n, int64_t k,
+                        float alpha, const void *A, int64_t lda,
+                        const void *B, int64_t ldb,
+                        float beta, void *C, int64_t ldc,
+                        char transA, char transB, hgemm_dtype_t out_dtype,
+                        hgemm_compute_t compute, cudaStream_t stream);
+
 /* Host-buffer variant: A, B and C are HOST pointers (page-locked memory gives
  * full copy/compute overlap; pageable memory works but serialises the copies),
  * same meaning, layout and quick-return rules as hgemm().  The call is
@@ -80,10 +108,16 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k,
  * hgemm_host_workspace_size(...) bytes (it holds the device copies of A, B
  * and C).  The problem is processed in column panels of op(B)/C: panel j's
  * host->device copy, GEMM and device->host copy run on three internal
- * streams so the transfers of one panel overlap the GEMM of another.
- * `stream` orders the whole call after prior work on it (0 = legacy stream).
+ * streams so the transfers of one panel overlap the GEMM of another; the
+ * first panel's GEMM is cut into row pieces of op(A) that start as soon as
+ * their rows of A have arrived.  Calls on one device are serialised (the
+ * pipeline streams are per device); calls on different devices run
+ * concurrently.  `stream` orders the whole call after prior work on it
+ * (0 = legacy stream).
  * Errors: HGEMM_ERR_INVALID_VALUE as for hgemm(), also for a NULL or too
- * small workspace; HGEMM_ERR_CUDA for copy/launch failures. */
+ * small workspace; HGEMM_ERR_CUDA for copy/launch failures.  An error after
+ * the first copy was enqueued returns only once the internal streams have
+ * drained, so no copy touches the caller's host buffers afterwards. */
 size_t hgemm_host_workspace_size(int64_t m, int64_t n, int64_t k, char transA, char transB,
                                  hgemm_dtype_t out_dtype);
 hgemm_status_t hgemm_host(int64_t m, int64_t n, int64_t k,

@@ -18,6 +18,7 @@ HEADER = os.path.join(_ROOT, "include", "hgemm.h")
 HGEMM_OUT_F16 = 0
 HGEMM_OUT_F32 = 1
 HGEMM_KERNEL = {"auto": 0, "simt": 1, "tc1": 2, "tc2": 3, "splitk": 4, "stream": 5}
+HGEMM_COMPUTE = {"f32": 0, "f16": 1}
 
 _lib = None
 
@@ -63,6 +64,9 @@ def load_library():
     lib.hgemm.argtypes = [i64, i64, i64, f32, vp, i64, vp, i64, f32, vp, i64,
                           ctypes.c_char, ctypes.c_char, ctypes.c_int, vp]
     lib.hgemm.restype = ctypes.c_int
+    lib.hgemm_ex.argtypes = [i64, i64, i64, f32, vp, i64, vp, i64, f32, vp, i64,
+                             ctypes.c_char, ctypes.c_char, ctypes.c_int, ctypes.c_int, vp]
+    lib.hgemm_ex.restype = ctypes.c_int
     lib.hgemm_status_string.argtypes = [ctypes.c_int]
     lib.hgemm_status_string.restype = ctypes.c_char_p
     lib.hgemm_set_config.argtypes = [ctypes.POINTER(_Config)]
@@ -175,6 +179,19 @@ def hgemm(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", transB="N",
     code = lib.hgemm(int(m), int(n), int(k), float(alpha), _ptr(A), int(lda), _ptr(B), int(ldb),
                      float(beta), _ptr(C), int(ldc), transA.encode()[:1], transB.encode()[:1],
                      _out_code(out_dtype), _stream(stream))
+    _check(code)
+
+
+def hgemm_ex(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", transB="N",
+             out_dtype=HGEMM_OUT_F16, compute="f32", stream=None):
+    """hgemm() with an explicit accumulation type (include/hgemm.h hgemm_ex):
+    compute "f32" (FP32 accumulation, as hgemm) or "f16" (FP16 accumulation on the
+    tensor cores, the paper's HMMA.1688.F16 mode; FP16 output only)."""
+    lib = load_library()
+    comp = HGEMM_COMPUTE[compute] if isinstance(compute, str) else int(compute)
+    code = lib.hgemm_ex(int(m), int(n), int(k), float(alpha), _ptr(A), int(lda), _ptr(B), int(ldb),
+                        float(beta), _ptr(C), int(ldc), transA.encode()[:1], transB.encode()[:1],
+                        _out_code(out_dtype), comp, _stream(stream))
     _check(code)
 
 

@@ -27,6 +27,12 @@ def sources():
                   + [os.path.join(ROOT, "include", "hgemm.h")])
 
 
+def units():
+    """Translation units of libhgemm.so: the C ABI (hgemm_api.cu) and one TU per kernel
+    family (hgemm_inst_*.cu), compiled in parallel and linked into one library."""
+    return sorted(glob.glob(os.path.join(CSRC, "hgemm_*.cu")))
+
+
 def needs_build() -> bool:
     if not os.path.exists(LIB):
         return True
@@ -35,8 +41,11 @@ def needs_build() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
-    """Compile csrc/hgemm_api.cu into `out` (default: the in-tree libhgemm.so).
-    `defines` adds -D flags (experiment variants are built to other paths)."""
+    """Compile the TUs of csrc/ into `out` (default: the in-tree libhgemm.so), one nvcc
+    process per TU in parallel.  `defines` adds -D flags (experiment variants are built
+    to other paths)."""
+    from concurrent.futures import ThreadPoolExecutor
+    import tempfile
     target = out or LIB
     if not force and out is None and not defines and not needs_build():
         return LIB
@@ -44,12 +53,24 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     # HGEMM_WATCHDOG_CYCLES > 0 builds a debug library whose pipeline waits trap after that
     # many cycles (a deadlock becomes a launch error instead of a hung GPU).
     watchdog = os.environ.get("HGEMM_WATCHDOG_CYCLES", "0")
-    cmd = [NVCC, *ARCH, f"-DHGEMM_WATCHDOG_CYCLES={watchdog}ll", "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-shared",
-           "-I", os.path.join(ROOT, "include"), "-o", tmp, os.path.join(CSRC, "hgemm_api.cu")]
-    cmd[1:1] = [f"-D{d}" for d in defines]
+    flags = [*ARCH, *[f"-D{d}" for d in defines], f"-DHGEMM_WATCHDOG_CYCLES={watchdog}ll", "-O3", "-std=c++17",
+             "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-I", os.path.join(ROOT, "include")]
     if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-    subprocess.check_call(cmd)
+        flags.append("-Xptxas=-v")
+    with tempfile.TemporaryDirectory(prefix="hgemm_build_") as td:
+        objs = []
+
+        def compile_one(src):
+            obj = os.path.join(td, os.path.basename(src)[:-3] + ".o")
+            subprocess.check_call([NVCC, *flags, "-c", "-o", obj, src])
+            return obj
+        with ThreadPoolExecutor(max_workers=max(1, min(len(units()), os.cpu_count() or 1))) as ex:
+            objs = list(ex.map(compile_one, units()))
+        # export the C ABI only (the hgi:: internals shared between the TUs stay local)
+        vs = os.path.join(td, "exports.map")
+        with open(vs, "w") as f:
+            f.write("{ global: hgemm*; local: *; };\n")
+        subprocess.check_call([NVCC, *ARCH, "-shared", "-Xlinker", f"--version-script={vs}", "-o", tmp, *objs])
     os.replace(tmp, target)
     return target
 

@@ -18,33 +18,37 @@
 #include <mutex>
 
 #include "../../include/hgemm.h"
+#include "hgemm_internal.cuh"
 #include "hgemm_simt.cuh"
-#include "hgemm_splitk.cuh"
 #include "hgemm_stream.cuh"
-#include "hgemm_tc.cuh"
+
+
+// ----------------------------------------------------------------- shared state (hgemm_internal.cuh)
+namespace hgi {
+std::atomic<int64_t> g_launches{0};
+extern const bool g_pdl = [] {
+  const char *e = std::getenv("HGEMM_PDL");
+  return !(e && e[0] == '0');
+}();
+thread_local bool t_half_used = false;
+}  // namespace hgi
 
 namespace {
 
 using hg::TcParams;
-using hg::TcShape;
+using hgi::DeviceInfo;
+using hgi::g_launches;
+using hgi::g_pdl;
+using hgi::kMaxDevices;
+using hgi::t_half_used;
 
 // ----------------------------------------------------------------- device info
-struct DeviceInfo {
-  bool init = false;
-  bool ok = false;
-  int num_sms = 0;
-  int max_clusters_2sm = 0;  // filled lazily per kernel (same for all 2-SM instantiations)
-};
-constexpr int kMaxDevices = 64;
 DeviceInfo g_dev[kMaxDevices];
 std::mutex g_mu;
 
 hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0};
 hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0};
-std::atomic<int64_t> g_launches{0};
 std::atomic<unsigned long long *> g_probe{nullptr};
-// programmatic dependent launch of the tensor-core kernels (HGEMM_PDL=0 disables it: experiments)
-thread_local bool t_half_used = false;  // the last tile launch of this thread used the half-tile tail
 // experiment knobs, read once at load time (never per call)
 int env_int(const char *name, int dflt) {
   const char *e = std::getenv(name);
@@ -55,10 +59,6 @@ const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pa
 const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster groups along N
 const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hints
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
-const bool g_pdl = [] {
-  const char *e = std::getenv("HGEMM_PDL");
-  return !(e && e[0] == '0');
-}();
 
 bool device_info(int dev, DeviceInfo &out) {
   if (dev < 0 || dev >= kMaxDevices) return false;
@@ -163,6 +163,9 @@ bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer
   return true;
 }
 
+}  // namespace
+
+namespace hgi {
 // ----------------------------------------------------------------- stream-K
 // Stream-K plan for `tiles` tiles of `nkb` k-blocks on `units` persistent
 // clusters: whole waves minus one run data-parallel, the rest is split into
@@ -175,7 +178,7 @@ bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer
 // more SMs gains nothing by itself; the FP32 fixup traffic and the lost
 // lockstep between clusters sharing panels cost about a third of a wave.  Stream-K
 // pays off only when the last data-parallel wave is nearly empty.
-inline double sk_overhead_waves(int64_t nkb) { return 0.35 + 4.0 / static_cast<double>(nkb); }
+double sk_overhead_waves(int64_t nkb) { return 0.35 + 4.0 / static_cast<double>(nkb); }
 int sk_plan(int64_t tiles, int64_t units, int64_t nkb, int mode) {
   if (mode == 1 || units <= 1 || tiles % units == 0 || nkb < 2) return -1;
   const int64_t dp = tiles > units ? (tiles / units - 1) * units : 0;
@@ -227,192 +230,11 @@ bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags)
   return true;
 }
 
-// ----------------------------------------------------------------- TC launch
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC, bool AG = false>
-hgemm_status_t launch_tc(const CUtensorMap &ta, const CUtensorMap &tb, const CUtensorMap &td, const TcParams &p0,
-                         int dev, const DeviceInfo &di, int max_ctas, int sk_mode, bool *sk_used,
-                         cudaStream_t stream) {
-  using S = TcShape<BN, CG, OUT_F32>;
-  constexpr int THREADS = S::THREADS + (AG ? 32 : 0);  // + the all-gather copy warp
-  const int ht_mode = sk_mode >> 4;  // hgemm_config_t::half_tail, packed above the stream-K mode
-  sk_mode &= 15;
-  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC, AG>;
-  static int attr_done[kMaxDevices] = {};
-  static int max_clusters[kMaxDevices] = {};
-  if (!attr_done[dev]) {
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, S::SMEM_BYTES) != cudaSuccess)
-      return HGEMM_ERR_CUDA;
-    if (CG == 2) {
-      cudaLaunchConfig_t qc = {};
-      qc.gridDim = dim3(CG * MC * (di.num_sms / (CG * MC)));
-      qc.blockDim = dim3(THREADS);
-      qc.dynamicSmemBytes = S::SMEM_BYTES;
-      cudaLaunchAttribute qa[1];
-      qa[0].id = cudaLaunchAttributeClusterDimension;
-      qa[0].val.clusterDim.x = CG * MC;
-      qa[0].val.clusterDim.y = 1;
-      qa[0].val.clusterDim.z = 1;
-      qc.attrs = qa;
-      qc.numAttrs = 1;
-      int n = 0;
-      if (cudaOccupancyMaxActiveClusters(&n, kern, &qc) != cudaSuccess || n <= 0) n = di.num_sms / (CG * MC);
-      max_clusters[dev] = n;
-    } else {
-      max_clusters[dev] = di.num_sms;
-    }
-    attr_done[dev] = 1;
-  }
-  const int tiles = p0.num_m_tiles * p0.num_n_tiles;
-  int units = max_clusters[dev];
-  if (max_ctas > 0) units = std::max(1, std::min(units, max_ctas / (CG * MC)));
-  int clusters = std::min(tiles, units);
-  TcParams p = p0;
-  p.dp_tiles = tiles;
-  p.sk_u0 = p.sk_units = 0;
-  p.sk_ws = nullptr;
-  p.sk_flags = nullptr;
-  p.n_half = 0;
-  *sk_used = false;
-  // half-tile tail (512-wide tiles): a last wave of r <= units/2 tiles runs as 2r
-  // 256-wide items, i.e. in about half the time
-  bool half_tail = false;
-  if (BN == 512 && CG == 2 && MC == 1 && !AG && ht_mode != 1 && sk_mode != 2) {
-    const int r = tiles % units;
-    if (r > 0 && 2 * r <= units && (ht_mode == 2 || tiles / units >= 4)) {
-      p.n_half = r;
-      p.dp_tiles = tiles + r;
-      clusters = std::min(tiles + r, units);
-      half_tail = true;
-    }
-  }
-  t_half_used = half_tail;
-  if (MC == 1 && !AG && !half_tail) {
-    const int dp = sk_plan(tiles, units, p.num_k_blocks, sk_mode);
-    float *ws = nullptr;
-    int *flags = nullptr;
-    if (dp >= 0 && units * CG * MC <= di.num_sms && sk_workspace(dev, stream, di.num_sms, &ws, &flags)) {
-      p.dp_tiles = dp;
-      p.sk_u0 = static_cast<int64_t>(dp) * p.num_k_blocks;
-      p.sk_units = static_cast<int64_t>(tiles - dp) * p.num_k_blocks;
-      p.sk_ws = ws;
-      p.sk_flags = flags;
-      clusters = units;
-      *sk_used = true;
-    }
-  }
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(clusters * CG * MC);
-  cfg.blockDim = dim3(THREADS);
-  cfg.dynamicSmemBytes = S::SMEM_BYTES;
-  cfg.stream = stream;
-  cudaLaunchAttribute attr[2];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = CG * MC;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  // programmatic dependent launch: the prologue overlaps the previous kernel's tail
-  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
-  cfg.attrs = attr;
-  cfg.numAttrs = 2;
-  if (cudaLaunchKernelEx(&cfg, kern, ta, tb, td, p) != cudaSuccess) return HGEMM_ERR_CUDA;
-  g_launches.fetch_add(1, std::memory_order_relaxed);
-  return HGEMM_SUCCESS;
-}
+}  // namespace hgi
 
-template <int BN, int CG, int MC = 1>
-hgemm_status_t dispatch_tc_layout(bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
-                                  const CUtensorMap &td, const TcParams &p, int dev, const DeviceInfo &di,
-                                  int max_ctas, int sk_mode, bool *sk_used, cudaStream_t s) {
-#define HG_CASE(AM, BM_, F)                                                               \
-  if (a_mn == AM && b_mn == BM_ && f32 == F)                                              \
-    return launch_tc<BN, CG, AM, BM_, F, MC>(ta, tb, td, p, dev, di, max_ctas, sk_mode, sk_used, s);
-  HG_CASE(false, false, false)
-  HG_CASE(false, false, true)
-  HG_CASE(false, true, false)
-  HG_CASE(false, true, true)
-  HG_CASE(true, false, false)
-  HG_CASE(true, false, true)
-  HG_CASE(true, true, false)
-  HG_CASE(true, true, true)
-#undef HG_CASE
-  return HGEMM_ERR_INVALID_VALUE;
-}
-
-// fused all-gather kernels: CTA pairs, op(A) K-major (transA = 'T')
-template <int BN>
-hgemm_status_t dispatch_tc_ag(bool a_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
-                              const CUtensorMap &td, const TcParams &p, int dev, const DeviceInfo &di, int max_ctas,
-                              bool *sk_used, cudaStream_t s) {
-  if (!a_mn && !f32) return launch_tc<BN, 2, false, false, false, 1, true>(ta, tb, td, p, dev, di, max_ctas, 1, sk_used, s);
-  if (!a_mn && f32) return launch_tc<BN, 2, false, false, true, 1, true>(ta, tb, td, p, dev, di, max_ctas, 1, sk_used, s);
-  if (a_mn && !f32) return launch_tc<BN, 2, true, false, false, 1, true>(ta, tb, td, p, dev, di, max_ctas, 1, sk_used, s);
-  return launch_tc<BN, 2, true, false, true, 1, true>(ta, tb, td, p, dev, di, max_ctas, 1, sk_used, s);
-}
-
-// ----------------------------------------------------------------- split-K launch
-template <int BN, int SPL, bool A_MN, bool B_MN, bool OUT_F32>
-hgemm_status_t launch_splitk(const CUtensorMap &ta, const CUtensorMap &tb, const TcParams &p, int dev,
-                             cudaStream_t stream) {
-  using SH = hg::SkShape<BN, SPL>;
-  auto kern = hg::hgemm_splitk_kernel<BN, SPL, A_MN, B_MN, OUT_F32>;
-  static int attr_done[kMaxDevices] = {};
-  if (!attr_done[dev]) {
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SH::SMEM_BYTES) != cudaSuccess)
-      return HGEMM_ERR_CUDA;
-    if (SPL > 8 && cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess)
-      return HGEMM_ERR_CUDA;
-    attr_done[dev] = 1;
-  }
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(static_cast<unsigned>(p.num_m_tiles * p.num_n_tiles * SPL));
-  cfg.blockDim = dim3(192);
-  cfg.dynamicSmemBytes = SH::SMEM_BYTES;
-  cfg.stream = stream;
-  cudaLaunchAttribute attr[2];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = SPL;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
-  cfg.attrs = attr;
-  cfg.numAttrs = 2;
-  if (cudaLaunchKernelEx(&cfg, kern, ta, tb, p) != cudaSuccess) return HGEMM_ERR_CUDA;
-  g_launches.fetch_add(1, std::memory_order_relaxed);
-  return HGEMM_SUCCESS;
-}
-
-template <int BN, int SPL>
-hgemm_status_t dispatch_splitk_layout(bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
-                                      const TcParams &p, int dev, cudaStream_t s) {
-#define HG_SK(AM, BM_, F) \
-  if (a_mn == AM && b_mn == BM_ && f32 == F) return launch_splitk<BN, SPL, AM, BM_, F>(ta, tb, p, dev, s);
-  HG_SK(false, false, false)
-  HG_SK(false, false, true)
-  HG_SK(false, true, false)
-  HG_SK(false, true, true)
-  HG_SK(true, false, false)
-  HG_SK(true, false, true)
-  HG_SK(true, true, false)
-  HG_SK(true, true, true)
-#undef HG_SK
-  return HGEMM_ERR_INVALID_VALUE;
-}
-
-hgemm_status_t dispatch_splitk(int bn, int spl, bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta,
-                               const CUtensorMap &tb, const TcParams &p, int dev, cudaStream_t s) {
-  if (bn == 64) {
-    if (spl == 2) return dispatch_splitk_layout<64, 2>(a_mn, b_mn, f32, ta, tb, p, dev, s);
-    if (spl == 4) return dispatch_splitk_layout<64, 4>(a_mn, b_mn, f32, ta, tb, p, dev, s);
-    if (spl == 8) return dispatch_splitk_layout<64, 8>(a_mn, b_mn, f32, ta, tb, p, dev, s);
-  } else {
-    if (spl == 2) return dispatch_splitk_layout<128, 2>(a_mn, b_mn, f32, ta, tb, p, dev, s);
-    if (spl == 4) return dispatch_splitk_layout<128, 4>(a_mn, b_mn, f32, ta, tb, p, dev, s);
-    if (spl == 8) return dispatch_splitk_layout<128, 8>(a_mn, b_mn, f32, ta, tb, p, dev, s);
-  }
-  return HGEMM_ERR_INVALID_VALUE;
-}
+namespace {
+using hgi::sk_plan;
+using hgi::sk_overhead_waves;
 
 inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
@@ -438,13 +260,11 @@ template <int MT, bool F32>
 hgemm_status_t launch_stream(const CUtensorMap &ta, const CUtensorMap &tb, const hg::StreamParams &p, int grid,
                              int dev, cudaStream_t stream) {
   auto kern = hg::hgemm_stream_kernel<MT, F32>;
-  static int attr_done[kMaxDevices] = {};
-  if (!attr_done[dev]) {
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, hg::kStreamSmemBytes) !=
-        cudaSuccess)
-      return HGEMM_ERR_CUDA;
-    attr_done[dev] = 1;
-  }
+  static hgi::KernInit init;
+  std::call_once(init.once[dev], [&] {
+    init.err[dev] = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, hg::kStreamSmemBytes);
+  });
+  if (init.err[dev] != cudaSuccess) return HGEMM_ERR_CUDA;
   const uint32_t smem = p.stages * p.stage_bytes + 1024u /*align*/ + 512u /*barriers*/;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(static_cast<unsigned>(grid));
@@ -604,11 +424,12 @@ struct AgSpec {
 
 hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const void *A, int64_t lda,
                           const void *B, int64_t ldb, float beta, void *C, int64_t ldc, char transA, char transB,
-                          hgemm_dtype_t out_dtype, cudaStream_t stream, const AgSpec *ag) {
+                          hgemm_dtype_t out_dtype, cudaStream_t stream, const AgSpec *ag, bool acc16 = false) {
   // ---------------------------------------------------------- validation (no side effects)
   if (m < 0 || n < 0 || k < 0) return HGEMM_ERR_INVALID_VALUE;
   if (!(is_t(transA) || is_n(transA)) || !(is_t(transB) || is_n(transB))) return HGEMM_ERR_INVALID_VALUE;
   if (out_dtype != HGEMM_OUT_F16 && out_dtype != HGEMM_OUT_F32) return HGEMM_ERR_INVALID_VALUE;
+  if (acc16 && (out_dtype != HGEMM_OUT_F16 || ag)) return HGEMM_ERR_INVALID_VALUE;
   const bool tA = is_t(transA), tB = is_t(transB);
   if (lda < std::max<int64_t>(1, tA ? k : m)) return HGEMM_ERR_INVALID_VALUE;
   if (ldb < std::max<int64_t>(1, tB ? n : k)) return HGEMM_ERR_INVALID_VALUE;
@@ -655,14 +476,22 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
                      lda < (1ll << 36) && ldb < (1ll << 36) && ldc < (1ll << 36) && encode_fn() != nullptr;
   const bool want_simt = !ag && (cfg.kernel == HGEMM_KERNEL_SIMT);
   if (!tc_ok || want_simt) {
-    dim3 grid(static_cast<unsigned>(cdiv(m, 64)), static_cast<unsigned>(cdiv(n, 64)));
-    if (grid.y > 65535u) return HGEMM_ERR_INVALID_VALUE;
-    const __half *Ah = static_cast<const __half *>(A);
-    const __half *Bh = static_cast<const __half *>(B);
-    if (f32) hg::hgemm_simt_kernel<true><<<grid, 256, 0, stream>>>(m, n, k, alpha, Ah, lda, Bh, ldb, beta, C, ldc, tA, tB);
-    else hg::hgemm_simt_kernel<false><<<grid, 256, 0, stream>>>(m, n, k, alpha, Ah, lda, Bh, ldb, beta, C, ldc, tA, tB);
-    if (cudaPeekAtLastError() != cudaSuccess) return HGEMM_ERR_CUDA;
-    g_launches.fetch_add(1, std::memory_order_relaxed);
+    // grid.y is limited to 65535 blocks of 64 columns: wider problems run as several
+    // launches over column ranges (pointer offsets into op(B) and C)
+    constexpr int64_t kColsPerLaunch = 65535ll * 64;
+    for (int64_t j0 = 0; j0 < n; j0 += kColsPerLaunch) {
+      const int64_t nj = std::min(n - j0, kColsPerLaunch);
+      dim3 grid(static_cast<unsigned>(cdiv(m, 64)), static_cast<unsigned>(cdiv(nj, 64)));
+      const __half *Ah = static_cast<const __half *>(A);
+      const __half *Bh = static_cast<const __half *>(B);
+      if (Bh) Bh += tB ? j0 : j0 * ldb;
+      void *Cj = static_cast<char *>(C) + j0 * ldc * (f32 ? 4 : 2);
+      if (f32) hg::hgemm_simt_kernel<true, false><<<grid, 256, 0, stream>>>(m, nj, k, alpha, Ah, lda, Bh, ldb, beta, Cj, ldc, tA, tB);
+      else if (acc16) hg::hgemm_simt_kernel<false, true><<<grid, 256, 0, stream>>>(m, nj, k, alpha, Ah, lda, Bh, ldb, beta, Cj, ldc, tA, tB);
+      else hg::hgemm_simt_kernel<false, false><<<grid, 256, 0, stream>>>(m, nj, k, alpha, Ah, lda, Bh, ldb, beta, Cj, ldc, tA, tB);
+      if (cudaPeekAtLastError() != cudaSuccess) return HGEMM_ERR_CUDA;
+      g_launches.fetch_add(1, std::memory_order_relaxed);
+    }
     std::lock_guard<std::mutex> lk(g_mu);
     g_last = {HGEMM_KERNEL_SIMT, 0, 0, 0, 0};
     return HGEMM_SUCCESS;
@@ -674,7 +503,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   const bool b_mn = !tA;  // Bk = op(A):   'N' -> rows of Bk contiguous along N
 
   // ---------------------------------------------------------- HBM streaming (skinny, TN)
-  if (!ag && !a_mn && !b_mn && M <= 256 &&
+  if (!ag && !acc16 && !a_mn && !b_mn && M <= 256 &&
       ((cfg.kernel == HGEMM_KERNEL_STREAM) ||
        (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream(M, N, k, di.num_sms)))) {
     const int mt = M <= 128 ? 1 : 2;
@@ -723,7 +552,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   // streaming kernel then keeps op(A) (m <= 256 rows) resident as its UMMA A operand,
   // streams the rows of op(B)^T (K-contiguous for transB 'N') and stores D = C
   // transposed (column-major C, element (i, j) at C + j*ldc + i).
-  if (!ag && !a_mn && !b_mn && N <= 256 && M > 256 &&
+  if (!ag && !acc16 && !a_mn && !b_mn && N <= 256 && M > 256 &&
       ((cfg.kernel == HGEMM_KERNEL_STREAM) ||
        (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream_swapped(N, M, k, di.num_sms)))) {
     const int64_t Ms = N, Ns = M;  // the swapped problem: M' = m, N' = n
@@ -771,8 +600,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   {
     int sk_bn = 0, sk_spl = 0;
     bool use_sk = false;
-    if (ag) {
-      // the fused all-gather runs the persistent tile kernel only
+    if (ag || acc16) {
+      // the fused all-gather and FP16 accumulation run the persistent tile kernel only
     } else if (cfg.kernel == HGEMM_KERNEL_SPLITK) {
       use_sk = true;
       sk_bn = cfg.block_n ? cfg.block_n : (N <= 64 ? 64 : 128);
@@ -803,7 +632,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
       p.D = C;
       p.ldd = ldc;
       p.probe = g_probe.load(std::memory_order_relaxed);
-      const hgemm_status_t st = dispatch_splitk(sk_bn, sk_spl, a_mn, b_mn, f32, ta, tb, p, dev, stream);
+      const hgemm_status_t st = sk_bn == 64 ? hgi::dispatch_splitk64(sk_spl, a_mn, b_mn, f32, ta, tb, p, dev, stream)
+                                            : hgi::dispatch_splitk128(sk_spl, a_mn, b_mn, f32, ta, tb, p, dev, stream);
       if (st == HGEMM_SUCCESS) {
         std::lock_guard<std::mutex> lk(g_mu);
         g_last = {HGEMM_KERNEL_SPLITK, sk_bn, p.group_m, 0, sk_spl};
@@ -813,12 +643,13 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   }
 
   int cg = 2, bn = 512;
-  // the fused all-gather kernels exist for CTA pairs only
-  const int forced_cg = ag ? 2 : cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
+  // the fused all-gather and FP16-accumulate kernels exist for CTA pairs only
+  const int forced_cg = (ag || acc16) ? 2 : cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
   // stream-K is off under the fused all-gather (its work items do not follow the chunk order)
-  // stream-K mode with hgemm_config_t::half_tail packed above it (launch_tc, choose_tc)
-  const int skm = (ag ? 1 : cfg.stream_k) | (cfg.half_tail << 4);
-  if (forced_cg && cfg.block_n && !(ag && cfg.block_n == 128)) { cg = forced_cg; bn = cfg.block_n; }
+  // and with FP16 accumulation (no FP32 partials); stream-K mode with hgemm_config_t::half_tail
+  // packed above it (launch_tc, choose_tc)
+  const int skm = ((ag || acc16) ? 1 : cfg.stream_k) | (cfg.half_tail << 4);
+  if (forced_cg && cfg.block_n && !((ag || acc16) && cfg.block_n == 128)) { cg = forced_cg; bn = cfg.block_n; }
   else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, skm, cg, bn);
   const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
   // MC = 2: two CTA pairs per cluster share (multicast) the Bk half-boxes
@@ -826,7 +657,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   // the two pairs' pipelines; built only with -DHGEMM_ENABLE_MC)
   int mc = 1;
 #ifdef HGEMM_ENABLE_MC
-  if (cg == 2 && !ag) {
+  if (cg == 2 && !ag && !acc16) {
     mc = g_env_mc == 2 ? 2 : 1;  // experiments
   }
 #endif
@@ -884,26 +715,12 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   p.D = C;
   p.ldd = ldc;
 
-  hgemm_status_t st;
   bool sk_used = false;
-#ifdef HGEMM_ENABLE_MC
-  if (cg == 2 && bn == 512 && mc == 2)
-    st = dispatch_tc_layout<512, 2, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
-  else if (cg == 2 && mc == 2)
-    st = dispatch_tc_layout<256, 2, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
-  else
-#endif
-  if (ag)
-    st = bn == 512 ? dispatch_tc_ag<512>(a_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, &sk_used, stream)
-                   : dispatch_tc_ag<256>(a_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, &sk_used, stream);
-  else if (cg == 2 && bn == 512)
-    st = dispatch_tc_layout<512, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
-  else if (cg == 2)
-    st = dispatch_tc_layout<256, 2>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
-  else if (bn == 256)
-    st = dispatch_tc_layout<256, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
-  else
-    st = dispatch_tc_layout<128, 1>(a_mn, b_mn, f32, ta, tb, td, p, dev, di, cfg.max_ctas, skm, &sk_used, stream);
+  const hgi::TcLaunch L = {&ta, &tb, &td, &p, dev, &di, cfg.max_ctas, skm, &sk_used, stream};
+  hgemm_status_t st;
+  if (cg == 2 && bn == 512) st = hgi::dispatch_tc512(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
+  else if (cg == 2) st = hgi::dispatch_tc256x2(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
+  else st = hgi::dispatch_tc1(bn, a_mn, b_mn, f32, L);
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);
     g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0, sk_used ? 2 : 1,
@@ -922,6 +739,14 @@ hgemm_status_t hgemm(int64_t m, int64_t n, int64_t k, float alpha, const void *A
   return hgemm_core(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA, transB, out_dtype, stream, nullptr);
 }
 
+hgemm_status_t hgemm_ex(int64_t m, int64_t n, int64_t k, float alpha, const void *A, int64_t lda, const void *B,
+                        int64_t ldb, float beta, void *C, int64_t ldc, char transA, char transB,
+                        hgemm_dtype_t out_dtype, hgemm_compute_t compute, cudaStream_t stream) {
+  if (compute != HGEMM_COMPUTE_F32 && compute != HGEMM_COMPUTE_F16) return HGEMM_ERR_INVALID_VALUE;
+  return hgemm_core(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA, transB, out_dtype, stream, nullptr,
+                    compute == HGEMM_COMPUTE_F16);
+}
+
 }  // extern "C"
 
 // ===================================================================== host-buffer path
@@ -934,7 +759,8 @@ struct HostPipe {
   cudaEvent_t ev_in[kEv] = {}, ev_comp[kEv] = {}, ev_start = nullptr;
 };
 HostPipe g_pipe[kMaxDevices];
-std::mutex g_pipe_mu;
+std::mutex g_pipe_mu;                     // creation of the per-device pipeline
+std::mutex g_pipe_call_mu[kMaxDevices];   // one hgemm_host call at a time per device
 
 inline int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 
@@ -1005,62 +831,97 @@ hgemm_status_t hgemm_host(int64_t m, int64_t n, int64_t k, float alpha, const vo
       P.init = true;
     }
   }
-  std::lock_guard<std::mutex> call_lk(g_pipe_mu);  // the pipeline streams/events serve one call at a time
+  // the pipeline streams/events of a device serve one call at a time (calls on other devices proceed)
+  std::lock_guard<std::mutex> call_lk(g_pipe_call_mu[dev]);
   const int esz = f32 ? 4 : 2;
   uint8_t *ws = static_cast<uint8_t *>(workspace);
   const int64_t lda_d = align_up(std::max<int64_t>(L.a_rows, 1), 8);
   const int64_t ldb_d = align_up(std::max<int64_t>(L.b_rows, 1), 8);
   const int64_t ldc_d = align_up(std::max<int64_t>(m, 1), f32 ? 4 : 8);
-  void *dA = ws + L.off_a, *dB = ws + L.off_b, *dC = ws + L.off_c;
+  uint8_t *dA = ws + L.off_a, *dB = ws + L.off_b, *dC = ws + L.off_c;
+  const uint8_t *hA = static_cast<const uint8_t *>(A), *hB = static_cast<const uint8_t *>(B);
+  uint8_t *hC = static_cast<uint8_t *>(C);
 
-  // panel width: >= 1024 columns, at most kEv panels, a multiple of 256
-  int64_t panels = std::min<int64_t>(HostPipe::kEv - 1, std::max<int64_t>(1, n / 1024));
-  if (panels > 8) panels = 8;
-  int64_t pw = align_up(cdiv(n, panels), 256);
+  // Column panels of op(B)/C (>= 1024 columns, at most 8, a multiple of 256 wide).  The
+  // first panel's GEMM is further cut into row pieces of op(A) (multiples of 256 rows) so
+  // that it starts once the first piece of A has arrived instead of all of A.
+  int64_t panels = std::min<int64_t>(8, std::max<int64_t>(1, n / 1024));
+  const int64_t pw = align_up(cdiv(n, panels), 256);
   panels = cdiv(n, pw);
+  const int64_t pieces = need_ab ? std::min<int64_t>(4, std::max<int64_t>(1, m / 2048)) : 1;
+  const int64_t ph = align_up(cdiv(m, pieces), 256);
+
+  // Once anything is enqueued, an error return first drains the internal streams: no
+  // copy may still read or write the caller's host buffers after the call returns.
+  auto fail = [&](hgemm_status_t st) {
+    cudaStreamSynchronize(P.s_in);
+    cudaStreamSynchronize(P.s_comp);
+    cudaStreamSynchronize(P.s_out);
+    return st;
+  };
+  int step = 0;
+  // one pipeline step: (H2D copies already on s_in) -> GEMM of C[r0:r1, n0:n1] on s_comp -> D2H on s_out
+  auto gemm_step = [&](int64_t r0, int64_t r1, int64_t n0, int64_t n1) -> hgemm_status_t {
+    if (cudaEventRecord(P.ev_in[step], P.s_in) != cudaSuccess) return HGEMM_ERR_CUDA;
+    if (cudaStreamWaitEvent(P.s_comp, P.ev_in[step], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
+    const uint8_t *dAi = dA + (tA ? r0 * lda_d : r0) * 2;
+    const uint8_t *dBj = dB + (tB ? n0 : n0 * ldb_d) * 2;
+    uint8_t *dCij = dC + (r0 + n0 * ldc_d) * esz;
+    const hgemm_status_t st = hgemm(r1 - r0, n1 - n0, k, alpha, dAi, lda_d, dBj, ldb_d, beta, dCij, ldc_d, transA,
+                                    transB, out_dtype, P.s_comp);
+    if (st != HGEMM_SUCCESS) return st;
+    if (cudaEventRecord(P.ev_comp[step], P.s_comp) != cudaSuccess) return HGEMM_ERR_CUDA;
+    if (cudaStreamWaitEvent(P.s_out, P.ev_comp[step], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
+    if (cudaMemcpy2DAsync(hC + (r0 + n0 * ldc) * esz, ldc * esz, dCij, ldc_d * esz, (r1 - r0) * esz, n1 - n0,
+                          cudaMemcpyDeviceToHost, P.s_out) != cudaSuccess)
+      return HGEMM_ERR_CUDA;
+    ++step;
+    return HGEMM_SUCCESS;
+  };
+  auto copy_b = [&](int64_t n0, int64_t n1) -> bool {  // op(B)[:, n0:n1] (+ C[:, n0:n1] when beta != 0)
+    const int64_t w = n1 - n0;
+    if (need_ab) {
+      // B columns (transB 'N') or B rows (transB 'T')
+      const size_t width = static_cast<size_t>(tB ? w : L.b_rows) * 2;
+      const size_t height = static_cast<size_t>(tB ? L.b_cols : w);
+      if (cudaMemcpy2DAsync(dB + (tB ? n0 : n0 * ldb_d) * 2, ldb_d * 2, hB + (tB ? n0 : n0 * ldb) * 2, ldb * 2,
+                            width, height, cudaMemcpyHostToDevice, P.s_in) != cudaSuccess)
+        return false;
+    }
+    if (beta != 0.0f &&
+        cudaMemcpy2DAsync(dC + n0 * ldc_d * esz, ldc_d * esz, hC + n0 * ldc * esz, ldc * esz, m * esz, w,
+                          cudaMemcpyHostToDevice, P.s_in) != cudaSuccess)
+      return false;
+    return true;
+  };
 
   if (cudaEventRecord(P.ev_start, stream) != cudaSuccess) return HGEMM_ERR_CUDA;
   if (cudaStreamWaitEvent(P.s_in, P.ev_start, 0) != cudaSuccess) return HGEMM_ERR_CUDA;
-  if (need_ab) {
-    if (cudaMemcpy2DAsync(dA, lda_d * 2, A, lda * 2, L.a_rows * 2, L.a_cols, cudaMemcpyHostToDevice, P.s_in) !=
-        cudaSuccess)
-      return HGEMM_ERR_CUDA;
-  }
-  for (int64_t j = 0; j < panels; ++j) {
-    const int64_t n0 = j * pw, n1 = std::min(n, n0 + pw), w = n1 - n0;
+  if (!copy_b(0, std::min(n, pw))) return fail(HGEMM_ERR_CUDA);
+  for (int64_t i = 0; i < pieces; ++i) {
+    const int64_t r0 = i * ph, r1 = std::min(m, r0 + ph);
+    if (r0 >= r1) break;
     if (need_ab) {
-      // op(B)[:, n0:n1]: B columns (transB 'N') or B rows (transB 'T')
-      const uint8_t *src = static_cast<const uint8_t *>(B) + (tB ? n0 : n0 * ldb) * 2;
-      uint8_t *dst = static_cast<uint8_t *>(dB) + (tB ? n0 : n0 * ldb_d) * 2;
-      const size_t width = static_cast<size_t>(tB ? w : L.b_rows) * 2;
-      const size_t height = static_cast<size_t>(tB ? L.b_cols : w);
-      if (cudaMemcpy2DAsync(dst, ldb_d * 2, src, ldb * 2, width, height, cudaMemcpyHostToDevice, P.s_in) !=
-          cudaSuccess)
-        return HGEMM_ERR_CUDA;
+      // op(A)[r0:r1, :]: stored columns r0..r1 (transA 'T') or rows r0..r1 of every column ('N')
+      const size_t width = static_cast<size_t>(tA ? L.a_rows : r1 - r0) * 2;
+      const size_t height = static_cast<size_t>(tA ? r1 - r0 : L.a_cols);
+      if (cudaMemcpy2DAsync(dA + (tA ? r0 * lda_d : r0) * 2, lda_d * 2, hA + (tA ? r0 * lda : r0) * 2, lda * 2,
+                            width, height, cudaMemcpyHostToDevice, P.s_in) != cudaSuccess)
+        return fail(HGEMM_ERR_CUDA);
     }
-    if (beta != 0.0f) {
-      if (cudaMemcpy2DAsync(static_cast<uint8_t *>(dC) + n0 * ldc_d * esz, ldc_d * esz,
-                            static_cast<const uint8_t *>(C) + n0 * ldc * esz, ldc * esz, m * esz, w,
-                            cudaMemcpyHostToDevice, P.s_in) != cudaSuccess)
-        return HGEMM_ERR_CUDA;
-    }
-    if (cudaEventRecord(P.ev_in[j], P.s_in) != cudaSuccess) return HGEMM_ERR_CUDA;
-    if (cudaStreamWaitEvent(P.s_comp, P.ev_in[j], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
-    const void *dBj = static_cast<const uint8_t *>(dB) + (tB ? n0 : n0 * ldb_d) * 2;
-    void *dCj = static_cast<uint8_t *>(dC) + n0 * ldc_d * esz;
-    const hgemm_status_t st = hgemm(m, w, k, alpha, dA, lda_d, dBj, ldb_d, beta, dCj, ldc_d, transA, transB,
-                                    out_dtype, P.s_comp);
-    if (st != HGEMM_SUCCESS) return st;
-    if (cudaEventRecord(P.ev_comp[j], P.s_comp) != cudaSuccess) return HGEMM_ERR_CUDA;
-    if (cudaStreamWaitEvent(P.s_out, P.ev_comp[j], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
-    if (cudaMemcpy2DAsync(static_cast<uint8_t *>(C) + n0 * ldc * esz, ldc * esz, dCj, ldc_d * esz, m * esz, w,
-                          cudaMemcpyDeviceToHost, P.s_out) != cudaSuccess)
-      return HGEMM_ERR_CUDA;
+    const hgemm_status_t st = gemm_step(r0, r1, 0, std::min(n, pw));
+    if (st != HGEMM_SUCCESS) return fail(st);
+  }
+  for (int64_t j = 1; j < panels; ++j) {
+    const int64_t n0 = j * pw, n1 = std::min(n, n0 + pw);
+    if (!copy_b(n0, n1)) return fail(HGEMM_ERR_CUDA);
+    const hgemm_status_t st = gemm_step(0, m, n0, n1);
+    if (st != HGEMM_SUCCESS) return fail(st);
   }
   // make `stream` observe the end of the pipeline (events recorded on it bracket the whole call)
-  if (cudaEventRecord(P.ev_comp[HostPipe::kEv - 1], P.s_out) != cudaSuccess) return HGEMM_ERR_CUDA;
-  if (cudaStreamWaitEvent(stream, P.ev_comp[HostPipe::kEv - 1], 0) != cudaSuccess) return HGEMM_ERR_CUDA;
-  if (cudaStreamSynchronize(P.s_out) != cudaSuccess) return HGEMM_ERR_CUDA;
+  if (cudaEventRecord(P.ev_comp[HostPipe::kEv - 1], P.s_out) != cudaSuccess) return fail(HGEMM_ERR_CUDA);
+  if (cudaStreamWaitEvent(stream, P.ev_comp[HostPipe::kEv - 1], 0) != cudaSuccess) return fail(HGEMM_ERR_CUDA);
+  if (cudaStreamSynchronize(P.s_out) != cudaSuccess) return fail(HGEMM_ERR_CUDA);
   return HGEMM_SUCCESS;
 }
 
@@ -1069,11 +930,15 @@ hgemm_status_t hgemm_host(int64_t m, int64_t n, int64_t k, float alpha, const vo
 // ============================================================================
 // Sharded path: all-gather of op(A) fused with the GEMM (include/hgemm.h;
 // BASELINE.json north_star (3), DESIGN.md "Fused
-// all-gather").  The copy engines pull the peers' rows of op(A) over NVLink
-// into the local gather buffer chunk by chunk and raise one flag per chunk;
-// the persistent GEMM kernel (already running) waits per tile for the chunks
-// it reads.  No SM is spent on the transfer and no NCCL kernel has to share
-// the SMs with the persistent GEMM.
+// all-gather").  An extra copy warp in every CTA of the persistent GEMM kernel
+// pulls the peers' rows of op(A) over NVLink (16-B loads from P2P-mapped peer
+// memory, 16 in flight per lane) into the local gather buffer, one ~64 KB copy
+// unit at a time from a shared work index, and counts finished units per
+// chunk; the TMA producer waits per tile for the chunks it reads.  The copy
+// warp costs issue slots and registers next to the epilogue warps of its SM;
+// the copy engines were rejected (a same-device cudaMemcpyAsync can run as a
+// kernel that never becomes resident next to the persistent GEMM),
+// and no NCCL kernel has to share the SMs with the GEMM.
 namespace {
 
 bool plan_args_ok(int64_t m, const int64_t *row_splits, int32_t world, int32_t rank, int64_t chunk_rows) {

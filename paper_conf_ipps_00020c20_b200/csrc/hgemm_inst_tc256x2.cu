@@ -1,0 +1,18 @@
+// Instantiations of the persistent tile kernel, CTA pair (cta_group::2), 256 x 256 pair tile
+// (double-buffered accumulators): all layouts, the fused all-gather variants and the
+// FP16-accumulate variants.
+#include "hgemm_internal.cuh"
+
+namespace hgi {
+
+hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_mn, bool f32, const TcLaunch &L) {
+#ifdef HGEMM_ENABLE_MC
+  if (mc == 2) return dispatch_tc_layout<256, 2, 2>(a_mn, b_mn, f32, L);
+#endif
+  (void)mc;
+  if (ag) return dispatch_tc_ag<256>(a_mn, f32, L);
+  if (acc16) return f32 ? HGEMM_ERR_INVALID_VALUE : dispatch_tc_acc16<256>(a_mn, b_mn, L);
+  return dispatch_tc_layout<256, 2, 1>(a_mn, b_mn, f32, L);
+}
+
+}  // namespace hgi

@@ -22,7 +22,11 @@ __device__ __forceinline__ void store_c(void *C, int64_t idx, float v) {
 }
 
 // 64 x 64 output tile per 256-thread block, 4 x 4 outputs per thread, K step 16.
-template <bool OUT_F32>
+// ACC16 (hgemm_ex HGEMM_COMPUTE_F16, FP16 output): an FP16 accumulator (the paper's
+// FP16-accumulate mode, P:98 / P:350) updated once per 16-deep K step, like one
+// tcgen05.mma kind::f16 K = 16 step: the step's 16 products are summed in FP32 and
+// the accumulator is rounded to FP16 after adding them.
+template <bool OUT_F32, bool ACC16 = false>
 __global__ void __launch_bounds__(256) hgemm_simt_kernel(int64_t m, int64_t n, int64_t k, float alpha,
                                                          const __half *__restrict__ A, int64_t lda,
                                                          const __half *__restrict__ B, int64_t ldb, float beta,
@@ -34,6 +38,16 @@ __global__ void __launch_bounds__(256) hgemm_simt_kernel(int64_t m, int64_t n, i
   const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
   float acc[4][4] = {};
   for (int64_t p0 = 0; p0 < k; p0 += 16) {
+    float acc0[4][4];  // ACC16: the accumulator before this K step
+    if constexpr (ACC16) {
+#pragma unroll
+      for (int r = 0; r < 4; ++r)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          acc0[r][c] = acc[r][c];
+          acc[r][c] = 0.f;
+        }
+    }
     for (int e = threadIdx.x; e < 16 * 64; e += 256) {
       const int pp = transA ? (e & 15) : (e >> 6);
       const int ii = transA ? (e >> 4) : (e & 63);
@@ -60,6 +74,12 @@ __global__ void __launch_bounds__(256) hgemm_simt_kernel(int64_t m, int64_t n, i
       for (int r = 0; r < 4; ++r)
 #pragma unroll
         for (int c = 0; c < 4; ++c) acc[r][c] = fmaf(a[r], b[c], acc[r][c]);
+    }
+    if constexpr (ACC16) {
+#pragma unroll
+      for (int r = 0; r < 4; ++r)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) acc[r][c] = __half2float(__float2half_rn(acc0[r][c] + acc[r][c]));
     }
     __syncthreads();
   }

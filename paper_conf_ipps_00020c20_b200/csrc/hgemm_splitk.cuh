@@ -5,12 +5,17 @@
 // of the cluster accumulates k-blocks [r*nkb/S, (r+1)*nkb/S) with
 // tcgen05.mma (cta_group::1) into its own TMEM.  The S partial accumulators
 // are then reduced through distributed shared memory, deterministically:
-// CTA r owns the column slice [r*BN/S, (r+1)*BN/S); every CTA pushes each
-// slice of its FP32 partial into the owner's shared memory (remote
-// st.shared::cluster), the cluster synchronises once, and each owner sums
-// its S received slices in split order 0..S-1 (fixed order => run-to-run
-// bitwise reproducible), applies alpha/beta and stores its slice of D.  No
-// global workspace, no atomics.
+// CTA r owns the column slice [r*BN/S, (r+1)*BN/S); every CTA stages the
+// slices of its FP32 partial it does not own in its (then idle) smem ring and
+// sends each warp's 32 rows of a slice to the owner with ONE bulk copy
+// (cp.async.bulk shared::cta -> shared::cluster) that completes on the owner's
+// receive mbarrier; each owner waits for its (S-1) x 128 x BN/S FP32 values,
+// sums the S slices in split order 0..S-1 (its own from registers; fixed
+// order => run-to-run bitwise reproducible), applies alpha/beta and stores its
+// slice of D.  No global workspace, no atomics, no cluster barrier between
+// the mainloop and the reduction (the first version pushed 16-B remote stores
+// and synchronised the cluster: 2.4 us from the last MMA to the reduction on
+// the LSTM-gate shapes, profiles/r01b/trace_splitk_lstm.log).
 //
 // Paper mapping: the blocked algorithm of Alg. 1 with the K loop
 // (line 6) divided among S thread blocks; the grid of SVI-A.2 is
@@ -41,6 +46,7 @@ struct SkShape {
   static_assert(S == 2 || S == 4 || S == 8, "S");
   static_assert(SLICE % 8 == 0, "slice");
   static_assert(STAGES >= 2, "stages");
+  static_assert(PART_BYTES <= STAGES * STAGE_BYTES, "reduction staging in the smem ring");
 };
 
 // Receive buffer of the owner CTA: [S sources][128 rows][SLICE FP32], the
@@ -96,7 +102,8 @@ __global__ void __launch_bounds__(192, 1)
   uint64_t *full = reinterpret_cast<uint64_t *>(part + SH::PART_BYTES);
   uint64_t *empty = full + STAGES;
   uint64_t *tfull = empty + STAGES;
-  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tfull + 1);
+  uint64_t *rbar = tfull + 1;  // receive barrier: (S-1) slices of 128 x SLICE FP32 from the peers
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(rbar + 1);
 
   const uint32_t warp = warp_id();
   const uint32_t lane = lane_id();
@@ -131,6 +138,10 @@ __global__ void __launch_bounds__(192, 1)
         mbar_init(&empty[s], 1);
       }
       mbar_init(tfull, 1);
+      mbar_init(rbar, 1);
+      // the peers' bulk copies complete their bytes on rbar (possibly before this arrival:
+      // the transaction count may run negative until the expectation is registered)
+      mbar_arrive_expect_tx(rbar, (S - 1) * 128u * SH::SLICE * 4u);
       fence_mbarrier_init();
     }
     __syncwarp();
@@ -139,6 +150,10 @@ __global__ void __launch_bounds__(192, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
+  // Cluster barrier, split: every thread arrives now (its barriers are initialised); a
+  // thread waits only before its first access to a peer's shared memory (the epilogue's
+  // bulk copies) or, for the producer / MMA warps, before exiting.
+  cluster_arrive();
   const uint32_t tmem_base = *tmem_slot;
   if (threadIdx.x == 0) SK_TRACE(1);
   griddep_wait();  // PDL: the prologue above overlapped the previous kernel; C is read right below
@@ -220,17 +235,21 @@ __global__ void __launch_bounds__(192, 1)
       else mbar_arrive(tfull);  // empty K range: the partial is zero
     }
   } else {
-    // ------------------------------------------------------------ epilogue warps: push partial slices
-    // CTA `rank` owns output columns [rank*SLICE, (rank+1)*SLICE) of the tile.
-    // Each CTA pushes the slice owned by CTA o into o's receive buffer at
-    // [rank][row][0..SLICE) (remote shared-memory stores, posted), so after
-    // one cluster barrier every owner reduces from its local shared memory.
+    // ------------------------------------------------------------ epilogue warps: split-K reduction
+    // CTA `rank` owns output columns [rank*SLICE, (rank+1)*SLICE) of the tile.  Each
+    // thread holds one tile row (its TMEM lane).  The slices owned by the peers are
+    // staged in the smem ring (free: every MMA has retired and no load is pending)
+    // in the owner's receive layout, then each warp sends its 32 rows of slice o with
+    // one bulk copy to owner o's buffer [rank][rows], completing on o's rbar.
+    constexpr int SLICE = SH::SLICE;
+    constexpr uint32_t SLAB = 128u * SLICE * 4u;  // one source's slice block: 128 rows x SLICE FP32
     const uint32_t quad = warp & 3u;
     const uint32_t prow = quad * 32u + lane;  // TMEM lane == tile row
+    const uint32_t stg = smem_u32(smem);      // staging: [owner][row][SLICE] (recv_off layout)
+    float own[SLICE];
     mbar_wait(tfull, 0);
     tc_fence_after();
     if (warp == 2 && lane == 0) SK_TRACE(4);
-    const uint32_t rbuf = smem_u32(part);
 #pragma unroll
     for (int c = 0; c < BN / 32; ++c) {
       uint32_t v[32];
@@ -244,32 +263,47 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
         const int colq = c * 32 + 4 * q;                  // first of these 4 tile columns
-        const uint32_t owner = static_cast<uint32_t>(colq / SH::SLICE);
-        const uint32_t within = static_cast<uint32_t>(colq % SH::SLICE) / 4;  // 16-B chunk in the slice
-        const uint32_t dst = mapa_shared(rbuf + recv_off(rank, prow, within), owner);
-        st_shared_cluster_v4(dst, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+        const uint32_t owner = static_cast<uint32_t>(colq / SLICE);
+        const uint32_t within = static_cast<uint32_t>(colq % SLICE) / 4;  // 16-B chunk in the slice
+        if (owner == rank) {
+#pragma unroll
+          for (int e = 0; e < 4; ++e) own[(colq % SLICE) + e] = __uint_as_float(v[4 * q + e]);
+        } else {
+          st_shared_v4(stg + owner * SLAB + recv_off(0u, prow, within), v[4 * q], v[4 * q + 1], v[4 * q + 2],
+                       v[4 * q + 3]);
+        }
       }
     }
     tc_fence_before();
-  }
+    fence_proxy_async_smem();  // the staged slices -> the bulk copies (async proxy)
+    __syncwarp();
+    cluster_wait();            // every peer's rbar is initialised before we copy into it
+    if (lane == 0) {
+      const uint32_t rows_off = quad * 32u * SLICE * 4u;  // this warp's 32 rows in a slice block
+#pragma unroll 1
+      for (uint32_t o = 0; o < static_cast<uint32_t>(S); ++o) {
+        if (o == rank) continue;
+        bulk_copy_s2cluster(mapa_shared(smem_u32(part) + rank * SLAB + rows_off, o), stg + o * SLAB + rows_off,
+                            32u * SLICE * 4u, mapa_shared(smem_u32(rbar), o));
+      }
+    }
+    if (warp == 2 && lane == 0) SK_TRACE(5);
 
-  // every slice has been pushed to its owner
-  cluster_sync();
-  if (threadIdx.x == 0) SK_TRACE(5);
-
-  if (warp >= 2) {
-    // ------------------------------------------------------------ local reduce + epilogue of this CTA's slice
-    constexpr int SLICE = SH::SLICE;
-    const uint32_t quad = warp & 3u;
-    const uint32_t prow = quad * 32u + lane;
+    // ------------------------------------------------------------ reduce + epilogue of this CTA's slice
     const int row = tm * BM + static_cast<int>(prow);
     const int col0 = tn * BN + static_cast<int>(rank) * SLICE;
     const uint32_t rbuf = smem_u32(part);
+    if constexpr (S > 1) mbar_wait(rbar, 0);  // the (S-1) peers' slices have landed
     float acc[SLICE];
 #pragma unroll
     for (int j = 0; j < SLICE; ++j) acc[j] = 0.0f;
 #pragma unroll
     for (int src = 0; src < S; ++src) {  // fixed summation order: split 0, 1, ..., S-1
+      if (static_cast<uint32_t>(src) == rank) {
+#pragma unroll
+        for (int j = 0; j < SLICE; ++j) acc[j] += own[j];
+        continue;
+      }
 #pragma unroll
       for (int q = 0; q < SLICE / 4; ++q) {
         const float4 v = ld_shared_f4(rbuf + recv_off(static_cast<uint32_t>(src), prow, q));
@@ -331,11 +365,11 @@ __global__ void __launch_bounds__(192, 1)
   }
 
   if (threadIdx.x == 64) SK_TRACE(6);
-  // No second cluster barrier: every remote (DSMEM) access of this kernel is a push
-  // that completed before the barrier above; the reduction reads local shared
-  // memory only, so a CTA may exit without waiting for its peers.
   __syncwarp();
-  __syncthreads();
+  if (warp < 2) cluster_wait();  // the producer / MMA warps' wait of the first cluster-barrier phase
+  // Second phase: a CTA may exit only after its peers have received its slices (the
+  // bulk copies read this CTA's staging area and complete only on the peers' rbar).
+  cluster_sync();
   if (threadIdx.x == 0) SK_TRACE(7);
   if (warp == 1) {
     tc_fence_after();

@@ -156,10 +156,10 @@ __device__ __forceinline__ uint64_t sdesc_mn_sw128(uint32_t saddr, uint32_t lbo)
   return d;
 }
 
-// Instruction descriptor for kind::f16: D FP32, A/B FP16, majorness, N, M.
-template <int M, int N, bool A_MN, bool B_MN>
+// Instruction descriptor for kind::f16: D FP32 (or FP16 with ACC16), A/B FP16, majorness, N, M.
+template <int M, int N, bool A_MN, bool B_MN, bool ACC16 = false>
 __host__ __device__ constexpr uint32_t make_idesc_f16() {
-  return (1u << 4)                                  // c_format = F32
+  return ((ACC16 ? 0u : 1u) << 4)                   // c_format: 1 = F32, 0 = F16 (the paper's HMMA.1688.F16)
          | (0u << 7) | (0u << 10)                   // a_format = b_format = F16
          | ((A_MN ? 1u : 0u) << 15) | ((B_MN ? 1u : 0u) << 16)
          | (static_cast<uint32_t>(N >> 3) << 17)    // N >> 3
@@ -188,6 +188,31 @@ __device__ __forceinline__ void tile_coords(int t, const TcParams &p, int &tm, i
   const int r = t - g * per_group;
   tm = first_m + r % gsz;
   tn = r / gsz;
+}
+
+// 64 accumulator columns of this thread's TMEM lane into v[0..63] (FP32 bit patterns
+// after acc_widen64).  ACC16 (c_format = F16, P:98 / P:350): every column holds an
+// FP16 value in its low 16 bits; one .pack::16b load brings the 64 columns as 32
+// half2 words, widened to FP32 (exactly) after tcgen05.wait::ld.
+template <bool ACC16>
+__device__ __forceinline__ void acc_ld64(uint32_t taddr, uint32_t (&v)[64]) {
+  if constexpr (ACC16) {
+    tmem_ld_32x32b_x32_pack16(taddr, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+  } else {
+    tmem_ld_32x32b_x32(taddr, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+    tmem_ld_32x32b_x32(taddr + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+  }
+}
+template <bool ACC16>
+__device__ __forceinline__ void acc_widen64(uint32_t (&v)[64]) {
+  if constexpr (ACC16) {
+#pragma unroll
+    for (int j = 31; j >= 0; --j) {  // in place, top down: v[j] is read before v[2j], v[2j+1] are written
+      const float2 f = __half22float2(*reinterpret_cast<const __half2 *>(&v[j]));
+      v[2 * j + 1] = __float_as_uint(f.y);
+      v[2 * j] = __float_as_uint(f.x);
+    }
+  }
 }
 
 __device__ __forceinline__ uint32_t pack_half2(float a, float b) {
@@ -303,17 +328,17 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
 // 5 + field for the first work item: 5 MMA done, 6 epilogue wake, 7 epilogue done.
 #define HG_CTRACE(it, field)                                                             \
   do {                                                                                   \
-    if (p.probe != nullptr && (it) == 0)                                                 \
+    if (p.probe != nullptr && (it) == 0 && blockIdx.x < 160)                            \
       p.probe[264 + 8 * blockIdx.x + 5 + (field)] = globaltimer_ns();                   \
   } while (0)
 #define HG_STAMP(slot)                                                                   \
   do {                                                                                   \
-    if (p.probe != nullptr) p.probe[264 + 8 * blockIdx.x + (slot)] = globaltimer_ns();   \
+    if (p.probe != nullptr && blockIdx.x < 160) p.probe[264 + 8 * blockIdx.x + (slot)] = globaltimer_ns();   \
   } while (0)
 // second region (producer start-up detail): p.probe[264 + 8*160 + 8*blockIdx.x + slot]
 #define HG_STAMP2(slot)                                                                  \
   do {                                                                                   \
-    if (p.probe != nullptr) p.probe[264 + 1280 + 8 * blockIdx.x + (slot)] = globaltimer_ns(); \
+    if (p.probe != nullptr && blockIdx.x < 160) p.probe[264 + 8 * 160 + 8 * blockIdx.x + (slot)] = globaltimer_ns(); \
   } while (0)
 #else
 #define HG_TRACE(it, field) \
@@ -389,7 +414,7 @@ __device__ __forceinline__ void ag_copy_warp(const TcParams &p, uint32_t lane) {
   }
 }
 
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC = 1, bool AG = false>
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC = 1, bool AG = false, bool ACC16 = false>
 __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 : 0), 1)
     hgemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmD, const TcParams p) {
@@ -408,7 +433,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
   constexpr uint32_t A_BYTES = S::A_BYTES;
   constexpr uint32_t B_HALF_BYTES = S::B_HALF_BYTES;
   constexpr uint32_t STAGE_BYTES = S::STAGE_BYTES;
-  constexpr uint32_t IDESC = make_idesc_f16<BM * CG, UMMA_N, A_MN, B_MN>();
+  constexpr uint32_t IDESC = make_idesc_f16<BM * CG, UMMA_N, A_MN, B_MN, ACC16>();
+  // FP16 accumulation (opt-in compute type, hgemm_ex): FP16 output, whole tiles only
+  static_assert(!ACC16 || (!OUT_F32 && MC == 1 && !AG), "ACC16: FP16 out, no multicast / all-gather");
   // Per-K=16 advance of the descriptor start address (in bytes).
   constexpr uint32_t A_KSTEP = A_MN ? 16 * 128 : 32;
   constexpr uint32_t B_KSTEP = B_MN ? 16 * 128 : 32;
@@ -924,9 +951,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             const int j = (half ? 0 : h * NB) + c;
             const int colt = h * UMMA_N + cgrp * EPI_COLS_W + c * EPI_COLS;
             uint32_t v[EPI_COLS];
-            tmem_ld_32x32b_x32(tbase + colt, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
-            if constexpr (EPI_COLS == 64) tmem_ld_32x32b_x32(tbase + colt + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+            if constexpr (EPI_COLS == 64) acc_ld64<ACC16>(tbase + colt, *reinterpret_cast<uint32_t(*)[64]>(&v[0]));
+            else tmem_ld_32x32b_x32(tbase + colt, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
             tmem_ld_wait();
+            if constexpr (EPI_COLS == 64) acc_widen64<ACC16>(*reinterpret_cast<uint32_t(*)[64]>(&v[0]));
             if (c == NB - 1) {
               tc_fence_before();
               __syncwarp();
@@ -1011,9 +1039,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
 #pragma unroll
           for (int b = 0; b < EPI_COLS_W / 64; ++b) {
             uint32_t v[64];
-            tmem_ld_32x32b_x32(tbase + c0 + b * 64, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
-            tmem_ld_32x32b_x32(tbase + c0 + b * 64 + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+            acc_ld64<ACC16>(tbase + c0 + b * 64, v);
             tmem_ld_wait();
+            acc_widen64<ACC16>(v);
             if (warp == 2 && lane == 0 && h == 0 && b == 0) HG_TRACE(it, 9);
             if constexpr (OUT_F32) {
 #pragma unroll
@@ -1084,9 +1112,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           // column within the tile (= TMEM column offset)
           const int colt = h * UMMA_N + cgrp * EPI_COLS_W + c * EPI_COLS;
           uint32_t v[64];
-          tmem_ld_32x32b_x32(tbase + colt, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
-          if constexpr (EPI_COLS == 64) tmem_ld_32x32b_x32(tbase + colt + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+          if constexpr (EPI_COLS == 64) acc_ld64<ACC16>(tbase + colt, v);
+          else tmem_ld_32x32b_x32(tbase + colt, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
           tmem_ld_wait();
+          if constexpr (EPI_COLS == 64) acc_widen64<ACC16>(v);
           if (c == EPI_COLS_W / EPI_COLS - 1) {
             // every TMEM read of this half is done: hand it back to the MMA warp
             tc_fence_before();

@@ -39,6 +39,40 @@ def integer_f16(rows: int, cols: int, seed: int, lo: int = -8, hi: int = 8) -> n
     return np.asfortranarray(x.T.astype(np.float16))
 
 
+def uniform_f16_blocked(rows: int, cols: int, seed: int, block: int = 4096, lo: float = -1.0,
+                        hi: float = 1.0, col0: int = 0, ncols: int | None = None) -> np.ndarray:
+    """Columns [col0, col0 + ncols) of a (rows, cols) uniform[lo, hi) FP16 matrix whose
+    column block b (columns [b*block, (b+1)*block)) is drawn by rng(seed * 100003 + b)
+    (SURVEY 8(e) "Inputs": the global matrix is defined block by block, so any slab of
+    it -- a rank's share at any world size -- is reproduced without drawing the rest).
+    Returns a Fortran-ordered (rows, ncols) array."""
+    ncols = cols - col0 if ncols is None else ncols
+    out = np.empty((rows, ncols), dtype=np.float16, order="F")
+    b0, b1 = col0 // block, (col0 + ncols + block - 1) // block
+    for b in range(b0, b1):
+        c0, c1 = b * block, min(cols, (b + 1) * block)
+        x = rng(seed * 100003 + b).random(size=(c1 - c0, rows), dtype=np.float32)
+        x *= np.float32(hi - lo)
+        x += np.float32(lo)
+        s0, s1 = max(c0, col0), min(c1, col0 + ncols)
+        out[:, s0 - col0:s1 - col0] = x[s0 - c0:s1 - c0].T.astype(np.float16)
+    return out
+
+
+def integer_f16_blocked(rows: int, cols: int, seed: int, lo: int, hi: int, block: int = 4096, col0: int = 0,
+                        ncols: int | None = None) -> np.ndarray:
+    """As uniform_f16_blocked, with integer values in [lo, hi] (exactly representable)."""
+    ncols = cols - col0 if ncols is None else ncols
+    out = np.empty((rows, ncols), dtype=np.float16, order="F")
+    b0, b1 = col0 // block, (col0 + ncols + block - 1) // block
+    for b in range(b0, b1):
+        c0, c1 = b * block, min(cols, (b + 1) * block)
+        x = rng(seed * 100003 + b).integers(lo, hi + 1, size=(c1 - c0, rows), dtype=np.int8)
+        s0, s1 = max(c0, col0), min(c1, col0 + ncols)
+        out[:, s0 - col0:s1 - col0] = x[s0 - c0:s1 - c0].T.astype(np.float16)
+    return out
+
+
 def to_colmajor(mat: np.ndarray, ld: int, fill=SENTINEL_F16) -> np.ndarray:
     """Flat column-major buffer of length ld*cols holding ``mat`` (rows <= ld)."""
     rows, cols = mat.shape

@@ -6,11 +6,14 @@ offsets with unchanged leading dimensions:
     op(B)[:, n0:n1]  ->  B + n0*ldb   (transB 'N')   or   B + n0   (transB 'T')
     C[:, n0:n1]      ->  C + n0*ldc
 No reduction is needed because K is not split, so each rank's slab is
-computed with exactly the single-GPU per-element arithmetic: the
-concatenation of the slabs is bitwise equal to the single-GPU result
-whenever the kernels keep whole tiles (stream-K off, hgemm_config_t
-stream_k = 1; with stream-K a tile split in k sums its FP32 partials in
-k order, which can round differently in the last place).
+computed with the single-GPU per-element arithmetic of whatever kernel the
+slab's shape selects.  The concatenation of the slabs is bitwise equal to
+the single-GPU result when every call runs the same tile kernel with whole
+tiles (e.g. hgemm_config_t kernel = tc2, a fixed block_n, stream_k = 1):
+with the automatic choice a narrow slab or a short panel can select split-K,
+the streaming kernel or stream-K, which sum the k-blocks of an element in a
+different grouping (results then agree within the north_star (4) bound, not
+bitwise).
 
 The one exchange step is the replication of A: an NCCL broadcast from the
 source rank over NVLink/NVSwitch (torch.distributed, backend "nccl" on
@@ -58,6 +61,29 @@ def broadcast_A(A, *, group=None, src=0):
         dist.broadcast(A, src=src, group=group)
 
 
+def order_after_current_stream(stream):
+    """Make `stream` wait for the work queued so far on torch's current CUDA stream.
+
+    torch.distributed's wait() (a synchronous broadcast, or Work.wait() of an async
+    one) orders the collective before later work on the CURRENT stream only; the
+    GEMM is enqueued on `stream`, which may be another stream, so it must wait on an
+    event recorded there.  `stream`: None (the current stream: nothing to do), an int
+    handle or a torch.cuda.Stream.  No-op without CUDA (the CPU tests)."""
+    if stream is None:
+        return
+    import torch
+    if not torch.cuda.is_available():
+        return
+    cur = torch.cuda.current_stream()
+    handle = int(stream) if isinstance(stream, int) else int(stream.cuda_stream)
+    if handle == int(cur.cuda_stream):
+        return
+    ev = torch.cuda.Event()
+    ev.record(cur)
+    target = torch.cuda.ExternalStream(handle) if isinstance(stream, int) else stream
+    target.wait_event(ev)
+
+
 def hgemm_sharded(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", transB="N",
                   out_dtype="f16", *, group=None, src=0, broadcast=True, local_slabs=False,
                   gemm=None, stream=None):
@@ -73,6 +99,8 @@ def hgemm_sharded(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, transA="N", tran
     world, rank = _world_rank(group)
     if broadcast:
         broadcast_A(A, group=group, src=src)
+        if world > 1:
+            order_after_current_stream(stream)   # the GEMM's stream sees the broadcast A
     n0, n1 = slab_bounds(n, world, rank)
     if gemm is None:
         from .binding import hgemm as gemm
@@ -99,7 +127,10 @@ def hgemm_sharded_overlapped(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, trans
     (in order on the communicator's stream); the GEMM of panel i
     (C[m0:m1, slab] = op(A)[m0:m1, :] op(B)[:, slab], a pointer offset into C)
     waits only for broadcast i, so it overlaps broadcasts i+1, i+2, ...
-    Every element is computed exactly as in the unpipelined path.
+    Each panel is its own hgemm() call: with a fixed tile kernel and whole tiles
+    (hgemm_config_t tc2 / block_n / stream_k = 1) every element is bitwise the
+    unpipelined result; with the automatic choice a short panel may select another
+    kernel (same north_star (4) bound, possibly different last bits).
     Returns this rank's (n0, n1)."""
     import torch.distributed as dist
     if transA not in ("T", "t"):
@@ -125,7 +156,8 @@ def hgemm_sharded_overlapped(m, n, k, alpha, A, lda, B, ldb, beta, C, ldc, trans
     for i in range(panels):
         p0, p1 = bounds[i], bounds[i + 1]
         if world > 1 and works[i] is not None:
-            works[i].wait()          # the compute stream waits for panel i only
+            works[i].wait()          # torch's current stream waits for panel i only ...
+            order_after_current_stream(stream)   # ... and so does the GEMM's stream
         if p1 > p0 and n1 > n0:
             gemm(p1 - p0, n1 - n0, k, alpha, _offset(A, p0 * lda * 2), lda, _offset(B, off_b), ldb, beta,
                  _offset(C, off_c + p0 * esz_c), ldc, transA, transB, out_dtype, stream)

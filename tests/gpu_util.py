@@ -51,7 +51,8 @@ class GpuCase:
         self.C_in = inputs.to_colmajor(np.asarray(C, dtype=cdt), self.ldc, fill=cdt(np.nan))
         self.Cmat = np.asarray(C, dtype=np.float64)
 
-    def run_gpu(self, repeat=1):
+    def run_gpu(self, repeat=1, compute=None):
+        """Run hgemm() (or hgemm_ex() with `compute` "f32" / "f16") on device copies."""
         from paper_conf_ipps_00020c20_b200 import binding
         torch = self.torch
         dA = torch.from_numpy(self.A.view(np.int16).copy()).cuda()
@@ -60,8 +61,12 @@ class GpuCase:
         outs = []
         for _ in range(repeat):
             dC = torch.from_numpy(cv.copy()).cuda()
-            binding.hgemm(self.m, self.n, self.k, self.alpha, dA, self.lda, dB, self.ldb, self.beta, dC,
-                          self.ldc, self.tA, self.tB, self.out)
+            if compute is None:
+                binding.hgemm(self.m, self.n, self.k, self.alpha, dA, self.lda, dB, self.ldb, self.beta, dC,
+                              self.ldc, self.tA, self.tB, self.out)
+            else:
+                binding.hgemm_ex(self.m, self.n, self.k, self.alpha, dA, self.lda, dB, self.ldb, self.beta, dC,
+                                 self.ldc, self.tA, self.tB, self.out, compute=compute)
             torch.cuda.synchronize()
             h = dC.cpu().numpy()
             if self.out == "f16":

@@ -128,3 +128,79 @@ def test_hgemm_torch_layouts(oracle_mod):
     want = 0.5 * exact + 2.0 * C0.double().cpu().numpy()
     bound = 1e-3 * (0.5 * absab + 2 * np.abs(C0.double().cpu().numpy())) + 2.0**-9 * np.abs(want) + 2**-24
     assert np.all(np.abs(C.double().cpu().numpy() - want) <= bound)
+
+
+# ---------------------------------------------------------------- BJ config 5: 32768^3, N-sharded
+def _cfg5_case(oracle_mod, n0, n1, *, integer=False, out="f16", seed=600, n_glob=32768):
+    """One rank's N-slab [n0, n1) of BASELINE.json configs[4] (m = n = k = 32768, TN, FP16 out),
+    generated block by block (inputs.uniform_f16_blocked) so the slab is exactly those
+    columns of the global B, run through hgemm() with the automatic choice (what
+    bench.py times per rank), checked on sampled entries + tile-edge rows/columns
+    against the oracle."""
+    import torch
+    from paper_conf_ipps_00020c20_b200 import binding
+    m = k = 32768
+    ns = n1 - n0
+    if integer:   # |C| <= ~6 sigma = 6*sqrt(k*4/9) ~ 720 < 2048: exact in FP32 and in FP16
+        At = inputs.integer_f16_blocked(k, m, seed, -1, 1)                       # stored A: k x m (op(A)^T)
+        Bs = inputs.integer_f16_blocked(k, n_glob, seed + 1, -1, 1, col0=n0, ncols=ns)
+    else:
+        At = inputs.uniform_f16_blocked(k, m, seed)
+        Bs = inputs.uniform_f16_blocked(k, n_glob, seed + 1, col0=n0, ncols=ns)
+    hA = At.reshape(-1, order="F")
+    hB = Bs.reshape(-1, order="F")
+    dA = torch.from_numpy(hA.view(np.int16)).cuda()
+    dB = torch.from_numpy(hB.view(np.int16)).cuda()
+    cdt = torch.float32 if out == "f32" else torch.float16
+    dC = torch.full((ns, m), float("nan"), dtype=cdt, device="cuda")
+    binding.set_config()
+    binding.hgemm(m, ns, k, 1.0, dA, k, dB, k, 0.0, dC, m, "T", "N", out)
+    torch.cuda.synchronize()
+    stats = binding.get_stats()
+    got = dC.cpu().numpy()
+    del dA, dB, dC
+    torch.cuda.empty_cache()
+    if out == "f16":
+        got = got.view(np.float16)
+    got = got.reshape(-1)                      # column-major C slab, ldc = m
+    ii, jj = _sample_indices(m, ns, count=2048, seed=seed)
+    _, r, ab = oracle_mod.hgemm_ref_entries(m, ns, k, 1.0, hA, k, hB, k, 0.0, None, m, "T", "N", out, ii, jj,
+                                            nthreads=oracle_mod.max_threads())
+    g = got[ii + jj * m].astype(np.float64)
+    if integer:
+        assert np.array_equal(g, r), f"{np.sum(g != r)} sampled entries differ (integer inputs must be exact)"
+    else:
+        bound = tolerance(r, ab, 1.0, 0.0, None, out, g)
+        bad = ~(np.abs(g - r) <= bound)
+        assert not bad.any(), f"{bad.sum()} sampled entries out of tolerance"
+        rel = float(np.max(np.abs(g - r) / np.maximum(ab, 1e-30)))
+        assert rel < 1e-5 + (2.0 ** -10 if out == "f16" else 0.0), rel
+    return stats
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("out", ["f16", "f32"])
+def test_cfg5_full_32768_one_gpu(oracle_mod, out):
+    """The whole 32768^3 problem on one GPU (the G = 1 point of config 5)."""
+    stats = _cfg5_case(oracle_mod, 0, 32768, out=out)
+    assert stats["last_kernel"] == "tc2", stats
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("g", [0, 7])
+def test_cfg5_g8_slab(oracle_mod, g):
+    """Rank g's slab at G = 8 (32768 x 4096 x 32768): the per-GPU problem of the 8-GPU run."""
+    stats = _cfg5_case(oracle_mod, 4096 * g, 4096 * (g + 1))
+    assert stats["last_kernel"] == "tc2", stats
+
+
+@pytest.mark.slow
+def test_cfg5_g8_slab_integer_exact(oracle_mod):
+    """Integer inputs in [-1, 1] at k = 32768 through the automatic multi-wave persistent path:
+    every partial sum is an integer < 2^24, so the sampled entries must be bit-exact."""
+    _cfg5_case(oracle_mod, 4096 * 3, 4096 * 4, integer=True)
+
+
+@pytest.mark.slow
+def test_cfg5_full_integer_exact(oracle_mod):
+    _cfg5_case(oracle_mod, 0, 32768, integer=True, out="f32")

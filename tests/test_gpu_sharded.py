@@ -1,5 +1,6 @@
 """Sharded path on one GPU (world size 1): the slab/panel bookkeeping around the
-CUDA kernels gives bitwise the single-call result (same per-element K order)."""
+CUDA kernels gives bitwise the single-call result (same per-element K order), and
+that result agrees with the CPU oracle on sampled entries (north_star (4))."""
 import numpy as np
 import pytest
 
@@ -7,16 +8,13 @@ pytestmark = pytest.mark.gpu
 
 
 def _setup(m, n, k, seed=0):
-    import torch
-    g = torch.Generator(device="cuda").manual_seed(seed)
-    A = (torch.rand(m, k, generator=g, device="cuda") * 2 - 1).half()   # stored k x m col-major: op(A) via 'T'
-    B = (torch.rand(n, k, generator=g, device="cuda") * 2 - 1).half()   # stored k x n col-major: 'N'
-    C0 = (torch.rand(n, m, generator=g, device="cuda") * 2 - 1).half()
+    from .test_gpu_allgather import _inputs
+    A, B, C0 = _inputs(m, n, k, k, "f16", 1.0, seed)   # host-drawn (inputs.py), copied to the device
     return A, B, C0
 
 
 @pytest.mark.parametrize("beta", [0.0, 1.0])
-def test_sharded_world1_equals_single_call(beta):
+def test_sharded_world1_equals_single_call(oracle_mod, beta):
     import torch
     from paper_conf_ipps_00020c20_b200 import binding, hgemm_sharded, hgemm_sharded_overlapped
     m, n, k = 2048, 1536, 1024
@@ -35,3 +33,5 @@ def test_sharded_world1_equals_single_call(beta):
     r = ref.cpu().numpy().view(np.uint16)
     assert np.array_equal(c1.cpu().numpy().view(np.uint16), r)
     assert np.array_equal(c2.cpu().numpy().view(np.uint16), r)
+    from .test_gpu_allgather import oracle_check
+    oracle_check(oracle_mod, m, n, k, A, k, B, k, beta, C0, c1, "f16")

@@ -24,7 +24,7 @@ for (m, n, k, beta) in [(256, 256, 256, 0.0), (4096, 1024, 4096, 1.0), (1024, 40
     B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
     C = (torch.rand(n, m, device="cuda") * 2 - 1).half()
     st = torch.zeros(2, dtype=torch.int64, device="cuda")
-    probe = torch.zeros(264 + 8 * 160, dtype=torch.int64, device="cuda")
+    probe = torch.zeros(264 + 2 * 8 * 160, dtype=torch.int64, device="cuda")
     s = torch.cuda.current_stream().cuda_stream
     for warm in (False, True):
         for i in range(4):

@@ -8,7 +8,8 @@ FP16 in / FP16 out, alpha = 1, beta = 0.  Each point: 3 warm-up runs, then
 the average of 10 runs timed with CUDA events (the paper's method),
 ours and cuBLAS (torch.mm, FP32 accumulation) alternating at every point.
 
-    python tools/paper_sweep.py [--square-step 256] [--rect-step 1024] [--out gpurun_out/sweep.jsonl]
+    python tools/paper_sweep.py [--square-step 256] [--rect-step 256] [--out gpurun_out/sweep.jsonl]
+                                [--md gpurun_out/sweep.md]
 """
 import argparse
 import json
@@ -23,7 +24,8 @@ from paper_conf_ipps_00020c20_b200 import binding  # noqa: E402
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--square-step", type=int, default=256)
-ap.add_argument("--rect-step", type=int, default=1024)
+ap.add_argument("--rect-step", type=int, default=256)
+ap.add_argument("--md", default=None, help="also write a markdown summary (per-shape mean / geomean / min)")
 ap.add_argument("--wmax", type=int, default=16384)
 ap.add_argument("--iters", type=int, default=10)
 ap.add_argument("--out", default="gpurun_out/paper_sweep.jsonl")
@@ -93,6 +95,36 @@ def main():
     rect = [r["speedup"] for r in recs if r["shape"] != "WxWxW"]
     print(f"square: mean speedup over cuBLAS {statistics.mean(sq):.3f} (min {min(sq):.3f}, max {max(sq):.3f}); "
           f"rectangular: mean {statistics.mean(rect):.3f} (min {min(rect):.3f}, max {max(rect):.3f})")
+    if args.md:
+        write_md(recs, args.md)
+
+
+def write_md(recs, path):
+    order = ["WxWxW", "2WxWxW", "Wx2WxW", "WxWx2W", "4WxWxW", "Wx4WxW", "WxWx4W"]
+    lines = ["| shape | points | mean ours/cuBLAS | geomean | min (W) | max (W) | mean ours TFLOP/s | mean cuBLAS TFLOP/s |",
+             "|---|---|---|---|---|---|---|---|"]
+    for sh in order:
+        rs = [r for r in recs if r["shape"] == sh]
+        if not rs:
+            continue
+        sp = [r["speedup"] for r in rs]
+        lo = min(rs, key=lambda r: r["speedup"])
+        hi = max(rs, key=lambda r: r["speedup"])
+        wkey = lambda r: r.get("W", r["m"])  # noqa: E731
+        lines.append(f"| {sh} | {len(rs)} | {statistics.mean(sp):.3f} | {statistics.geometric_mean(sp):.3f} | "
+                     f"{lo['speedup']:.3f} ({wkey(lo)}) | {hi['speedup']:.3f} ({wkey(hi)}) | "
+                     f"{statistics.mean(r['ours_tflops'] for r in rs):.1f} | "
+                     f"{statistics.mean(r['cublas_tflops'] for r in rs):.1f} |")
+    allsp = [r["speedup"] for r in recs]
+    lines.append(f"| all | {len(allsp)} | {statistics.mean(allsp):.3f} | {statistics.geometric_mean(allsp):.3f} | "
+                 f"{min(allsp):.3f} | {max(allsp):.3f} | | |")
+    lines += ["", "| shape | W | m | n | k | ours TFLOP/s | cuBLAS TFLOP/s | ours/cuBLAS | our kernel |",
+              "|---|---|---|---|---|---|---|---|---|"]
+    for r in recs:
+        lines.append(f"| {r['shape']} | {r.get('W', r['m'])} | {r['m']} | {r['n']} | {r['k']} | "
+                     f"{r['ours_tflops']:.1f} | {r['cublas_tflops']:.1f} | {r['speedup']:.3f} | {r['kernel']} |")
+    with open(path, "w") as f:
+        f.write("\n".join(lines) + "\n")
 
 
 if __name__ == "__main__":

@@ -36,7 +36,7 @@ for kern, bn in ([("tc2", 256), ("tc1", 256)] if not os.environ.get("HGEMM_LIB",
 if os.environ.get("HGEMM_LIB", "").endswith("trace.so"):
     for sk, mc in [(1, 0), (2, 0), (2, 130)]:
         binding.set_config("tc2", block_n=256, stream_k=sk, max_ctas=mc)
-        probe = torch.zeros(264 + 8 * 160, dtype=torch.int64, device="cuda")
+        probe = torch.zeros(264 + 2 * 8 * 160, dtype=torch.int64, device="cuda")
         for i in range(4):
             binding.set_probe(probe if i == 3 else None)
             binding.hgemm(m, n, k, 1.0, A, k, B, k, 0.0, C, m, "T", "N", "f16")

@@ -33,7 +33,7 @@ A = (torch.rand(m, k, device="cuda") * 2 - 1).half()
 B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
 C = (torch.rand(n, m, device="cuda") * 2 - 1).half()
 flush = torch.empty(64 * 1024 * 1024, device="cuda")
-probe = torch.zeros(264 + 8 * 160, dtype=torch.int64, device="cuda")
+probe = torch.zeros(264 + 2 * 8 * 160, dtype=torch.int64, device="cuda")
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 for i in range(6):
     if not a.warm:
