@@ -155,6 +155,10 @@ hgemm_status_t launch_tc(const TcLaunch &L) {
   attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 2;
+  if (CG * MC == 1 && (p.exp_flags & 16)) {  // experiment: plain (non-cluster) launch for 1-CTA "clusters"
+    cfg.attrs = attr + 1;
+    cfg.numAttrs = 1;
+  }
   if (cudaLaunchKernelEx(&cfg, kern, *L.ta, *L.tb, *L.td, p) != cudaSuccess) return HGEMM_ERR_CUDA;
   g_launches.fetch_add(1, std::memory_order_relaxed);
   return HGEMM_SUCCESS;

@@ -83,7 +83,9 @@ struct TcParams {
   // 1, accumulator half 0 only), so a last wave of R <= units/2 tiles takes half
   // the time.  Work items are numbered over tiles + n_half virtual items.
   int32_t n_half;
-  int32_t exp_flags;  // experiments (HGEMM_EXP): 1 = no ring staging for the last item, 2 = no C-load hold-back
+  int32_t exp_flags;  // experiments (HGEMM_EXP): 1 = no ring staging for the last item, 2 = no C-load hold-back,
+                      // 4 = wait for store completion before exit, 8 = no PDL trigger, 16 = no cluster
+                      // attribute for 1-CTA launches (host side)
 };
 
 // One unit of work of a cluster: k-blocks [kb0, kb1) of cluster tile `tile`.
@@ -620,7 +622,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         }
       }
       if (!cgo_sent) mbar_arrive(cgo);
-      griddep_launch_dependents();  // all loads issued: the next kernel may start its prologue
+      if (!(p.exp_flags & 8)) griddep_launch_dependents();  // all loads issued: the next kernel may start its prologue
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (leader CTA)
@@ -1043,7 +1045,16 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             tmem_ld_wait();
             acc_widen64<ACC16>(v);
             if (warp == 2 && lane == 0 && h == 0 && b == 0) HG_TRACE(it, 9);
-            if constexpr (OUT_F32) {
+            if (alpha == 1.0f) {  // alpha = 1 (the usual case): no multiply (bitwise the same result)
+              if constexpr (OUT_F32) {
+#pragma unroll
+                for (int j = 0; j < 64; ++j) pk[b * 64 + j] = v[j];
+              } else {
+#pragma unroll
+                for (int j = 0; j < 32; ++j)
+                  pk[b * 32 + j] = pack_half2(__uint_as_float(v[2 * j]), __uint_as_float(v[2 * j + 1]));
+              }
+            } else if constexpr (OUT_F32) {
 #pragma unroll
               for (int j = 0; j < 64; ++j) pk[b * 64 + j] = __float_as_uint(alpha * __uint_as_float(v[j]));
             } else {
@@ -1255,7 +1266,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
     // the staging buffers must have been read before the CTA exits; the stores'
     // global writes complete with the grid (the next kernel's griddepcontrol.wait
     // or stream order sees them)
-    if (lane == 0) bulk_wait_group_read<0>();
+    if (lane == 0) {
+      if (p.exp_flags & 4) bulk_wait_group<0>();  // experiment: the stores' global writes complete before exit
+      else bulk_wait_group_read<0>();
+    }
 #ifdef HGEMM_TRACE
     if (warp == 2 && lane == 0) HG_STAMP2(7);
 #endif

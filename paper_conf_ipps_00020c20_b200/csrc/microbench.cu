@@ -255,7 +255,84 @@ __global__ void empty_kernel(unsigned long long *dst, int touch_smem) {
   }
 }
 
+// Teardown probes (tools/teardown_probe.py): an otherwise empty kernel that
+// mode & 1: allocates and frees 512 TMEM columns (cta_group::1, or ::2 when the
+//           cluster has 2 CTAs), like the GEMM kernels;
+// mode & 2: issues one 4 KB bulk store (shared -> global) per warp and exits after
+//           its shared-memory read completed (the global write still in flight),
+//           like the GEMM epilogue;
+// mode & 4: executes griddepcontrol.launch_dependents early (PDL trigger).
+template <int CG>
+__global__ void teardown_kernel(int mode, uint8_t *gdst) {
+  using namespace hg;
+#if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
+  extern __shared__ uint8_t sm[];
+  __shared__ uint32_t slot;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (mode & 4) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  if ((mode & 1) && warp == 1) tmem_alloc<CG>(smem_u32(&slot), 512);
+  if (mode & 2) {
+    for (int i = threadIdx.x; i < 1024 * (blockDim.x / 32); i += blockDim.x) sm[i] = static_cast<uint8_t>(i);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if constexpr (CG == 2) cluster_sync();
+  tc_fence_after();
+  if ((mode & 2) && lane == 0) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    const size_t off = (static_cast<size_t>(blockIdx.x) * (blockDim.x / 32) + warp) * 4096;
+    bulk_store_1d(gdst + off, smem_u32(sm) + warp * 4096 % (1024 * (blockDim.x / 32)), 4096);
+    bulk_commit_group();
+    hg::bulk_wait_group_read<0>();
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  if constexpr (CG == 2) cluster_sync();
+  if ((mode & 1) && warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<CG>(slot, 512);
+  }
+#endif
+}
+
 extern "C" {
+
+int mb_teardown(int grid, int block, int smem, int cluster, int mode, int pdl, void *gdst, cudaStream_t s) {
+  static int attr = 0;
+  if (!attr) {
+    if (cudaFuncSetAttribute(teardown_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) !=
+            cudaSuccess ||
+        cudaFuncSetAttribute(teardown_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) !=
+            cudaSuccess)
+      return 2;
+    attr = 1;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute a[2];
+  int na = 0;
+  if (cluster > 0) {
+    a[na].id = cudaLaunchAttributeClusterDimension;
+    a[na].val.clusterDim.x = cluster;
+    a[na].val.clusterDim.y = 1;
+    a[na].val.clusterDim.z = 1;
+    ++na;
+  }
+  if (pdl) {
+    a[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    a[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+  }
+  cfg.attrs = a;
+  cfg.numAttrs = na;
+  cudaError_t e = cluster == 2 ? cudaLaunchKernelEx(&cfg, teardown_kernel<2>, mode, static_cast<uint8_t *>(gdst))
+                               : cudaLaunchKernelEx(&cfg, teardown_kernel<1>, mode, static_cast<uint8_t *>(gdst));
+  return e == cudaSuccess ? 0 : 1;
+}
 
 // Empty kernel with the tile kernel's launch shape (grid, block, dynamic smem,
 // cluster size): the fixed cost of such a launch, nothing else.

@@ -22,6 +22,7 @@ ap.add_argument("--m", type=int, default=8192)
 ap.add_argument("--warm", type=float, default=3.0)
 ap.add_argument("--iters", type=int, default=200)
 ap.add_argument("--order", default="ours,cublas,ours,cublas")
+ap.add_argument("--compute", default="f32", help="accumulation type of ours (f16: hgemm_ex FP16 accumulate)")
 args = ap.parse_args()
 m = n = k = args.m
 A = (torch.rand(m, k, device="cuda") * 2 - 1).half()    # op(A) rows, K-major: the paper's TN layout
@@ -31,7 +32,10 @@ torch.backends.cuda.matmul.allow_fp16_reduced_precision_reduction = False
 
 
 def ours():
-    binding.hgemm(m, n, k, 1.0, A, k, B, k, 0.0, C, m, "T", "N", "f16")
+    if args.compute == "f16":
+        binding.hgemm_ex(m, n, k, 1.0, A, k, B, k, 0.0, C, m, "T", "N", "f16", compute="f16")
+    else:
+        binding.hgemm(m, n, k, 1.0, A, k, B, k, 0.0, C, m, "T", "N", "f16")
 
 
 def cublas():

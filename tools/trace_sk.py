@@ -22,7 +22,7 @@ print(binding.get_stats())
 v = probe.cpu().view(-1).tolist()
 rows = [v[8 + 8 * b: 16 + 8 * b] for b in range(256) if v[8 + 8 * b]]
 t0 = min(r[0] for r in rows)
-names = ["start", "setup", "data0", "mma_issued", "tfull", "cl_sync1", "epi_done", "cl_sync2"]
+names = ["start", "setup", "data0", "mma_issued", "tfull", "sent", "epi_done", "end"]
 print("cta " + " ".join(f"{x:>10s}" for x in names))
 for b, r in enumerate(rows[:12]):
     print(f"{b:3d} " + " ".join(f"{(x - t0) if x else -1:10d}" for x in r))
