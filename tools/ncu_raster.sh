@@ -3,11 +3,11 @@
 M="gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sector_hit_rate.pct"
 for gm in 4 8 16 32; do
   timeout 200 ncu --metrics $M --clock-control none -k regex:hgemm_tc -s 3 -c 3 --csv --log-file gpurun_out/raster_gm$gm.csv \
-    python bench.py --steps 3 --warmup 3 --no-cpu --no-e2e --no-cublas --no-side --group-m $gm > /dev/null 2>&1
+    python bench.py --steps 3 --warmup 3 --no-cpu --no-e2e --no-cublas --no-side --no-strong --group-m $gm > /dev/null 2>&1
 done
 for gn in 4 8 16; do
   HGEMM_GROUP_N=$gn timeout 200 ncu --metrics $M --clock-control none -k regex:hgemm_tc -s 3 -c 3 --csv \
-    --log-file gpurun_out/raster_gn$gn.csv python bench.py --steps 3 --warmup 3 --no-cpu --no-e2e --no-cublas --no-side > /dev/null 2>&1
+    --log-file gpurun_out/raster_gn$gn.csv python bench.py --steps 3 --warmup 3 --no-cpu --no-e2e --no-cublas --no-side --no-strong > /dev/null 2>&1
 done
 python - <<'PY'
 import csv, glob, collections
