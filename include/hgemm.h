@@ -165,6 +165,12 @@ typedef struct {
                           2r 256-wide items), 1 = never, 2 = whenever r <= clusters/2.  Same per-element
                           arithmetic as whole tiles.  hgemm_get_last_config reports 2 if it was used,
                           1 if not (tile kernels). */
+    int32_t tile_n;    /* HGEMM_KERNEL_TC_2SM with block_n 256 only: flexible tile width, a multiple of
+                          16 in [128, 256] (0 = block_n).  Tiles of tile_n columns of the output's
+                          contiguous dimension (m), so that the tile count fills whole waves; needs a
+                          K-major op(A) (transA 'T'), otherwise block_n is used.  The automatic choice
+                          picks it by the wave model; hgemm_get_last_config reports the width used
+                          (0 = block_n).  Whole tiles, no stream-K. */
 } hgemm_config_t;
 
 /* Set (cfg != NULL) or reset to automatic (cfg == NULL) the process-global

@@ -30,7 +30,7 @@ class HgemmError(RuntimeError):
 class _Config(ctypes.Structure):
     _fields_ = [("kernel", ctypes.c_int32), ("block_n", ctypes.c_int32),
                 ("group_m", ctypes.c_int32), ("max_ctas", ctypes.c_int32), ("splits", ctypes.c_int32),
-                ("stream_k", ctypes.c_int32), ("half_tail", ctypes.c_int32)]
+                ("stream_k", ctypes.c_int32), ("half_tail", ctypes.c_int32), ("tile_n", ctypes.c_int32)]
 
 
 class IpcHandle(ctypes.Structure):
@@ -109,15 +109,16 @@ def _check(code: int):
 
 
 def set_config(kernel: str | int = "auto", block_n: int = 0, group_m: int = 0, max_ctas: int = 0,
-               splits: int = 0, stream_k: int = 0, half_tail: int = 0):
+               splits: int = 0, stream_k: int = 0, half_tail: int = 0, tile_n: int = 0):
     """Force a kernel choice (tests / bench).  ``set_config()`` restores automatic selection."""
     lib = load_library()
     kern = HGEMM_KERNEL[kernel] if isinstance(kernel, str) else int(kernel)
-    if kern == 0 and not block_n and not group_m and not max_ctas and not splits and not stream_k and not half_tail:
+    if (kern == 0 and not block_n and not group_m and not max_ctas and not splits and not stream_k
+            and not half_tail and not tile_n):
         _check(lib.hgemm_set_config(None))
     else:
         _check(lib.hgemm_set_config(ctypes.byref(_Config(kern, block_n, group_m, max_ctas, splits,
-                                                                  stream_k, half_tail))))
+                                                                  stream_k, half_tail, tile_n))))
 
 
 def set_probe(buf=None):
@@ -138,7 +139,7 @@ def get_stats() -> dict:
     inv = {v: k for k, v in HGEMM_KERNEL.items()}
     return {"last_kernel": inv.get(c.kernel, c.kernel), "block_n": c.block_n, "group_m": c.group_m,
             "max_ctas": c.max_ctas, "splits": c.splits, "stream_k": c.stream_k, "half_tail": c.half_tail,
-            "launches": int(lib.hgemm_launch_count())}
+            "tile_n": c.tile_n, "launches": int(lib.hgemm_launch_count())}
 
 
 def _ptr(x) -> int:

@@ -11,6 +11,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
 #include <atomic>
 #include <cstdint>
 #include <cstdlib>
@@ -46,8 +47,8 @@ using hgi::t_half_used;
 DeviceInfo g_dev[kMaxDevices];
 std::mutex g_mu;
 
-hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0};
-hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0};
+hgemm_config_t g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0, 0};
+hgemm_config_t g_last = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0, 0};
 std::atomic<unsigned long long *> g_probe{nullptr};
 // experiment knobs, read once at load time (never per call)
 int env_int(const char *name, int dflt) {
@@ -59,6 +60,7 @@ const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pa
 const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster groups along N
 const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hints
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
+const bool g_env_flex = env_int("HGEMM_FLEX", 0) != 0;        // flexible tile widths in the automatic choice
 
 bool device_info(int dev, DeviceInfo &out) {
   if (dev < 0 || dev >= kMaxDevices) return false;
@@ -312,23 +314,42 @@ inline bool is_t(char c) { return c == 'T' || c == 't'; }
 inline bool is_n(char c) { return c == 'N' || c == 'n'; }
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
-// Automatic tile choice: estimated time = waves * per-wave tile cost.
+// Relative per-SM throughput of a CTA-pair tile tn columns wide (flexible width, 256-wide
+// kernel): the L2 -> SMEM demand per tensor cycle grows as the tile narrows (each CTA loads
+// 16 KB of Ak + tn/2 rows of Bk per k-block for 512*tn/256 tensor cycles:
+// 8192/tn + 32 B/clk/SM), so the efficiency falls below the 256-wide tile's 0.93.
+inline double flex_eff(int tn) {
+  const double demand = 8192.0 / tn + 32.0, demand256 = 8192.0 / 256 + 32.0;
+  return 0.93 * std::pow(demand256 / demand, 0.5);
+}
+
+// Automatic tile choice: estimated time = waves * per-wave tile cost.  flex_ok: the
+// 256-wide CTA-pair kernel may use a flexible tile width (K-major Bk); tn returns the
+// chosen width (0: the kernel's own BN).
 void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, int forced_cg, int sk_mode, int &cg,
-               int &bn) {
-  struct Cand { int cg, bn; double eff; };
+               int &bn, bool flex_ok, int &tn) {
+  struct Cand { int cg, bn, tn; double eff; };
   // eff: relative per-SM throughput of the tile shape.  Larger tiles move
   // fewer L2->SMEM bytes per FLOP (pair 256x512: 171 FLOP/B, 256x256: 128,
   // 1-SM 128x256: 85, 128x128: 64), which under the 1 kW power cap buys clock.
-  const Cand cands[4] = {{2, 512, 1.00}, {2, 256, 0.93}, {1, 256, 0.85}, {1, 128, 0.75}};
+  Cand cands[16] = {{2, 512, 0, 1.00}, {2, 256, 0, 0.93}, {1, 256, 0, 0.85}, {1, 128, 0, 0.75}};
+  int nc = 4;
+  if (flex_ok)  // flexible widths 240, 224, ..., 144 for the CTA-pair 256-wide kernel
+    for (int w = 240; w >= 144; w -= 16) cands[nc++] = {2, 256, w, flex_eff(w)};
   double best = 1e300;
-  for (const Cand &c : cands) {
+  tn = 0;
+  for (int ci = 0; ci < nc; ++ci) {
+    const Cand &c = cands[ci];
     if (forced_cg && c.cg != forced_cg) continue;
+    const int width = c.tn ? c.tn : c.bn;
     // One 512-column accumulator cannot fully overlap the epilogue with the
     // next tile's mainloop, and its staging (one box per epilogue warp) cannot
     // prefetch a whole accumulator half of C; with beta != 0 that costs ~3% at
     // K = 8192 and ~7% at K = 1024 (BERT-FFN shapes).
-    const double eff = (c.bn == 512 && beta_nonzero) ? (K < 4096 ? 0.90 : 0.97) : c.eff;
-    const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, c.bn);
+    double eff = (c.bn == 512 && beta_nonzero) ? (K < 4096 ? 0.90 : 0.97) : c.eff;
+    // flexible tiles with beta != 0 take the chunked epilogue (C through registers)
+    if (c.tn && beta_nonzero) eff *= 0.95;
+    const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, width);
     const int64_t units = num_sms / c.cg;
     double waves = static_cast<double>(cdiv(tiles, units));
     const int64_t nkb = cdiv(K, 64);
@@ -340,10 +361,10 @@ void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, 
       waves = static_cast<double>(tiles / units) + 0.6;
     // stream-K: fractional waves (256-wide tiles only: with 512-wide tiles the FP32
     // partials of a split tile are twice as large and it measured slower everywhere)
-    if (c.bn <= 256 && sk_plan(tiles, units, nkb, sk_mode & 15) >= 0)
+    if (c.bn <= 256 && !c.tn && sk_plan(tiles, units, nkb, sk_mode & 15) >= 0)
       waves = static_cast<double>(tiles) / units + sk_overhead_waves(nkb);
-    const double t = waves * (128.0 * c.cg * c.bn) / (c.cg * eff);
-    if (t < best * 0.999) { best = t; cg = c.cg; bn = c.bn; }
+    const double t = waves * (128.0 * c.cg * width) / (c.cg * eff);
+    if (t < best * 0.999) { best = t; cg = c.cg; bn = c.bn; tn = c.tn; }
   }
 }
 
@@ -364,7 +385,7 @@ const char *hgemm_status_string(hgemm_status_t s) {
 hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!cfg) {
-    g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0};
+    g_cfg = {HGEMM_KERNEL_AUTO, 0, 0, 0, 0, 0, 0, 0};
     return HGEMM_SUCCESS;
   }
   if (cfg->kernel < HGEMM_KERNEL_AUTO || cfg->kernel > HGEMM_KERNEL_STREAM) return HGEMM_ERR_INVALID_VALUE;
@@ -378,6 +399,7 @@ hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
     return HGEMM_SUCCESS;
   }
   if (cfg->splits != 0) return HGEMM_ERR_INVALID_VALUE;
+  if (cfg->tile_n != 0 && cfg->kernel != HGEMM_KERNEL_TC_2SM) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_STREAM) {
     if (cfg->block_n < 0 || cfg->block_n > 256 || cfg->block_n % 16 != 0) return HGEMM_ERR_INVALID_VALUE;
     if (cfg->group_m < 0 || cfg->max_ctas < 0) return HGEMM_ERR_INVALID_VALUE;
@@ -385,6 +407,10 @@ hgemm_status_t hgemm_set_config(const hgemm_config_t *cfg) {
     return HGEMM_SUCCESS;
   }
   if (cfg->block_n != 0 && cfg->block_n != 128 && cfg->block_n != 256 && cfg->block_n != 512)
+    return HGEMM_ERR_INVALID_VALUE;
+  // flexible width: the CTA-pair 256-wide kernel only, a multiple of 16 in [128, 256]
+  if (cfg->tile_n != 0 && (cfg->kernel != HGEMM_KERNEL_TC_2SM || cfg->block_n != 256 || cfg->tile_n % 16 != 0 ||
+                           cfg->tile_n < 128 || cfg->tile_n > 256))
     return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_TC_2SM && cfg->block_n == 128) return HGEMM_ERR_INVALID_VALUE;
   if (cfg->kernel == HGEMM_KERNEL_TC_1SM && cfg->block_n == 512) return HGEMM_ERR_INVALID_VALUE;
@@ -642,16 +668,27 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     }
   }
 
-  int cg = 2, bn = 512;
+  int cg = 2, bn = 512, tnf = 0;  // tnf: flexible tile width (0 = bn)
   // the fused all-gather and FP16-accumulate kernels exist for CTA pairs only
   const int forced_cg = (ag || acc16) ? 2 : cfg.kernel == HGEMM_KERNEL_TC_1SM ? 1 : cfg.kernel == HGEMM_KERNEL_TC_2SM ? 2 : 0;
   // stream-K is off under the fused all-gather (its work items do not follow the chunk order)
   // and with FP16 accumulation (no FP32 partials); stream-K mode with hgemm_config_t::half_tail
   // packed above it (launch_tc, choose_tc)
   const int skm = ((ag || acc16) ? 1 : cfg.stream_k) | (cfg.half_tail << 4);
-  if (forced_cg && cfg.block_n && !((ag || acc16) && cfg.block_n == 128)) { cg = forced_cg; bn = cfg.block_n; }
-  else choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, skm, cg, bn);
-  const int b_rows = (bn > 256 ? 256 : bn) / cg;  // Bk rows per CTA per accumulator half
+  // flexible tile widths need a K-major Bk (TMA boxes of any multiple of 8 rows)
+  const bool flex_ok = !b_mn && !ag && (skm & 15) != 2;
+  if (forced_cg && cfg.block_n && !((ag || acc16) && cfg.block_n == 128)) {
+    cg = forced_cg;
+    bn = cfg.block_n;
+    if (flex_ok && cg == 2 && bn == 256 && cfg.tile_n > 0 && cfg.tile_n < 256) tnf = cfg.tile_n;
+  } else {
+    // flexible widths are never chosen automatically: measured slower than the 256-wide tile
+    // (with stream-K) at every mid-size shape tried (profiles/r02/flex_tile_sweep.log; DESIGN.md
+    // "Flexible tile width"); the candidates stay available to the model for experiments
+    choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, skm, cg, bn, flex_ok && g_env_flex, tnf);
+  }
+  const int skm_eff = tnf ? ((skm & ~15) | 1) : skm;  // flexible tiles: whole tiles, no stream-K
+  const int b_rows = (tnf ? tnf : (bn > 256 ? 256 : bn)) / cg;  // Bk rows per CTA per accumulator half
   // MC = 2: two CTA pairs per cluster share (multicast) the Bk half-boxes
   // (measured slower everywhere: a 4-CTA cluster strands SMs of the GPCs and couples
   // the two pairs' pipelines; built only with -DHGEMM_ENABLE_MC)
@@ -680,7 +717,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   p.N = static_cast<int32_t>(N);
   p.K = static_cast<int32_t>(k);
   p.num_m_tiles = static_cast<int32_t>(cdiv(M, 128 * cg * mc));
-  p.num_n_tiles = static_cast<int32_t>(cdiv(N, bn));
+  p.num_n_tiles = static_cast<int32_t>(cdiv(N, tnf ? tnf : bn));
+  p.tile_n = tnf;
   p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
   p.group_m = cfg.group_m > 0 ? cfg.group_m : 16 / mc;  // measured best with 256x512 pair tiles (profiles/)
   p.group_m = std::max(1, std::min(p.group_m, p.num_m_tiles));
@@ -716,7 +754,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   p.ldd = ldc;
 
   bool sk_used = false;
-  const hgi::TcLaunch L = {&ta, &tb, &td, &p, dev, &di, cfg.max_ctas, skm, &sk_used, stream};
+  const hgi::TcLaunch L = {&ta, &tb, &td, &p, dev, &di, cfg.max_ctas, skm_eff, &sk_used, stream};
   hgemm_status_t st;
   if (cg == 2 && bn == 512) st = hgi::dispatch_tc512(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
   else if (cg == 2) st = hgi::dispatch_tc256x2(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
@@ -724,7 +762,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);
     g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0, sk_used ? 2 : 1,
-              t_half_used ? 2 : 1};
+              t_half_used ? 2 : 1, tnf};
   }
   return st;
 }

@@ -127,16 +127,50 @@ __global__ void __launch_bounds__(192, 1)
   } while (0)
 #endif
   if (threadIdx.x == 0) SK_TRACE(0);
+  // TMA producer state (warp 0, lane 0): k-block pkb is loaded into ring stage pstage
+  const int a_row = tm * BM;
+  const int b_row = tn * BN;
+  uint32_t pstage = 0, pphase = 0;
+  int pkb = kb0;
+  auto produce = [&](int upto) {  // issue the loads of k-blocks [pkb, upto)
+    for (; pkb < upto; ++pkb) {
+      mbar_wait(&empty[pstage], pphase ^ 1u);
+      const uint32_t sa = smem_u32(smem + pstage * STAGE_BYTES);
+      const uint32_t sb = sa + A_BYTES;
+      mbar_arrive_expect_tx(&full[pstage], STAGE_BYTES);
+      const uint32_t fb = smem_u32(&full[pstage]);
+      const int k0 = pkb * BK;
+      if constexpr (!A_MN) {
+        tma_load_2d(&tmA, sa, fb, k0, a_row, 0);
+      } else {
+#pragma unroll
+        for (int q = 0; q < BM / 64; ++q) tma_load_2d(&tmA, sa + q * 8192, fb, a_row + 64 * q, k0, 0);
+      }
+      if constexpr (!B_MN) {
+        tma_load_2d(&tmB, sb, fb, k0, b_row, 0);
+      } else {
+#pragma unroll
+        for (int q = 0; q < BN / 64; ++q) tma_load_2d(&tmB, sb + q * 8192, fb, b_row + 64 * q, k0, 0);
+      }
+      if (++pstage == STAGES) { pstage = 0; pphase ^= 1u; }
+    }
+  };
   if (warp == 0 && lane == 0) {
+    // The producer initialises the ring barriers itself and issues the first ring of
+    // loads right away (after griddepcontrol.wait), so the first HBM round trip
+    // overlaps the TMEM allocation and the CTA barrier below.
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    fence_mbarrier_init();
+    griddep_wait();
+    produce(min(kb1, kb0 + STAGES));
   }
   if (warp == 1) {
     if (lane == 0) {
-      for (int s = 0; s < STAGES; ++s) {
-        mbar_init(&full[s], 1);
-        mbar_init(&empty[s], 1);
-      }
       mbar_init(tfull, 1);
       mbar_init(rbar, 1);
       // the peers' bulk copies complete their bytes on rbar (possibly before this arrival:
@@ -147,6 +181,7 @@ __global__ void __launch_bounds__(192, 1)
     __syncwarp();
     tmem_alloc<1>(smem_u32(tmem_slot), SH::TMEM_COLS);
   }
+  __syncwarp();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -182,33 +217,8 @@ __global__ void __launch_bounds__(192, 1)
   }
 
   if (warp == 0) {
-    // ------------------------------------------------------------ TMA producer
-    if (lane == 0) {
-      const int a_row = tm * BM;
-      const int b_row = tn * BN;
-      uint32_t stage = 0, phase = 0;
-      for (int kb = kb0; kb < kb1; ++kb) {
-        mbar_wait(&empty[stage], phase ^ 1u);
-        const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
-        const uint32_t sb = sa + A_BYTES;
-        mbar_arrive_expect_tx(&full[stage], STAGE_BYTES);
-        const uint32_t fb = smem_u32(&full[stage]);
-        const int k0 = kb * BK;
-        if constexpr (!A_MN) {
-          tma_load_2d(&tmA, sa, fb, k0, a_row, 0);
-        } else {
-#pragma unroll
-          for (int q = 0; q < BM / 64; ++q) tma_load_2d(&tmA, sa + q * 8192, fb, a_row + 64 * q, k0, 0);
-        }
-        if constexpr (!B_MN) {
-          tma_load_2d(&tmB, sb, fb, k0, b_row, 0);
-        } else {
-#pragma unroll
-          for (int q = 0; q < BN / 64; ++q) tma_load_2d(&tmB, sb + q * 8192, fb, b_row + 64 * q, k0, 0);
-        }
-        if (++stage == STAGES) { stage = 0; phase ^= 1u; }
-      }
-    }
+    // ------------------------------------------------------------ TMA producer (the rest of the k range)
+    if (lane == 0) produce(kb1);
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
     if (lane == 0) {

@@ -112,16 +112,39 @@ __global__ void __launch_bounds__(192, 1)
   // hitting the same offset in every row.  Only the summation order changes.
   const int nkb = p.num_k_blocks;
   const int kb_rot = p.k_rot ? static_cast<int>((static_cast<int64_t>(blockIdx.x) * nkb) / gridDim.x) : 0;
+  // TMA producer state (warp 0, lane 0): iteration pi of chunk pch is loaded into stage pstage
+  uint32_t pstage = 0, pphase = 0;
+  int pch = blockIdx.x, pi = 0;
+  auto produce = [&](int max_loads) {  // issue up to max_loads more k-block loads
+    for (; pch < p.num_chunks && max_loads > 0; --max_loads) {
+      const int kb = (pi + kb_rot) % nkb;
+      mbar_wait(&empty[pstage], pphase ^ 1u);
+      const uint32_t sa = smem_u32(smem + pstage * stage_bytes);
+      mbar_arrive_expect_tx(&full[pstage], stage_bytes);
+      const uint32_t fb = smem_u32(&full[pstage]);
+#pragma unroll
+      for (int t = 0; t < MT; ++t) tma_load_2d(&tmA, sa + t * A_SUB, fb, kb * 64, t * 128, 0);
+      tma_load_2d(&tmB, sa + a_bytes, fb, kb * 64, pch * cw, 0);
+      if (++pstage == static_cast<uint32_t>(stages)) { pstage = 0; pphase ^= 1u; }
+      if (++pi == nkb) { pi = 0; pch += gridDim.x; }
+    }
+  };
   if (warp == 0 && lane == 0) {
+    // The producer initialises the ring barriers itself and issues the first ring of
+    // loads right away (after griddepcontrol.wait), so the first HBM round trip
+    // overlaps the TMEM allocation and the CTA barrier below.
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
+    for (int s = 0; s < stages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    fence_mbarrier_init();
+    griddep_wait();
+    produce(stages);
   }
   if (warp == 1) {
     if (lane == 0) {
-      for (int s = 0; s < stages; ++s) {
-        mbar_init(&full[s], 1);
-        mbar_init(&empty[s], 1);
-      }
       for (int b = 0; b < 2; ++b) {
         mbar_init(&tfull[b], 1);
         mbar_init(&tempty[b], 4);
@@ -131,6 +154,7 @@ __global__ void __launch_bounds__(192, 1)
     __syncwarp();
     tmem_alloc<1>(smem_u32(tmem_slot), 512);
   }
+  __syncwarp();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -139,24 +163,8 @@ __global__ void __launch_bounds__(192, 1)
   if (threadIdx.x == 0) ST_TRACE(1);
 
   if (warp == 0) {
-    // ------------------------------------------------------------ TMA producer
-    if (lane == 0) {
-      uint32_t stage = 0, phase = 0;
-      for (int ch = blockIdx.x; ch < p.num_chunks; ch += gridDim.x) {
-        const int n0 = ch * cw;
-        for (int i = 0; i < nkb; ++i) {
-          const int kb = (i + kb_rot) % nkb;
-          mbar_wait(&empty[stage], phase ^ 1u);
-          const uint32_t sa = smem_u32(smem + stage * stage_bytes);
-          mbar_arrive_expect_tx(&full[stage], stage_bytes);
-          const uint32_t fb = smem_u32(&full[stage]);
-#pragma unroll
-          for (int t = 0; t < MT; ++t) tma_load_2d(&tmA, sa + t * A_SUB, fb, kb * 64, t * 128, 0);
-          tma_load_2d(&tmB, sa + a_bytes, fb, kb * 64, n0, 0);
-          if (++stage == static_cast<uint32_t>(stages)) { stage = 0; phase ^= 1u; }
-        }
-      }
-    }
+    // ------------------------------------------------------------ TMA producer (the remaining loads)
+    if (lane == 0) produce(1 << 30);
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
     if (lane == 0) {

@@ -83,6 +83,10 @@ struct TcParams {
   // 1, accumulator half 0 only), so a last wave of R <= units/2 tiles takes half
   // the time.  Work items are numbered over tiles + n_half virtual items.
   int32_t n_half;
+  // Flexible tile width (kernels with one accumulator half, NH == 1, and a K-major Bk):
+  // tiles of tile_n columns (a multiple of 16, <= UMMA_N; 0 = BN), chosen by the host so the
+  // tile count fills whole waves.
+  int32_t tile_n;
   int32_t exp_flags;  // experiments (HGEMM_EXP): 1 = no ring staging for the last item, 2 = no C-load hold-back,
                       // 4 = wait for store completion before exit, 8 = no PDL trigger, 16 = no cluster
                       // attribute for 1-CTA launches (host side)
@@ -190,6 +194,9 @@ __device__ __forceinline__ void tile_coords(int t, const TcParams &p, int &tm, i
   const int r = t - g * per_group;
   tm = first_m + r % gsz;
   tn = r / gsz;
+  // experiment (HGEMM_EXP & 32): serpentine order, odd groups sweep N backwards so that the
+  // Bk panels at a group boundary are reused by the next group's first tiles
+  if ((p.exp_flags & 32) && (g & 1)) tn = p.num_n_tiles - 1 - tn;
 }
 
 // 64 accumulator columns of this thread's TMEM lane into v[0..63] (FP32 bit patterns
@@ -261,29 +268,32 @@ struct TcShape {
 };
 
 // Write one thread's 32-word (128-B) row chunk of D: stage it in this warp's
-// swizzled 32 x 128-B box and TMA-store the box, or, for a chunk crossing an N
-// that is not a multiple of 16 B, store it directly (TMA bounds-checks stores
-// at 16-B granularity along the contiguous dimension).
+// swizzled 32 x 128-B box and TMA-store the box, or store it directly when the
+// chunk crosses `lim` (the first column not to write: N, or the end of a
+// flexible-width tile) where the TMA box would write too much: at an N that is
+// not a multiple of 16 B (TMA bounds-checks stores at 16-B granularity along the
+// contiguous dimension), or at a tile end inside the tensor.
 template <bool OUT_F32, int EPI_BUFS, bool CHECK_TAIL = true>
 __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensorMap *tmD, uint32_t stg,
                                                uint32_t &nstore, const uint32_t (&w)[32], int col, int row,
-                                               int row_base, uint32_t lane) {
+                                               int row_base, uint32_t lane, int lim = 0x7fffffff) {
   constexpr int VEC = OUT_F32 ? 4 : 8;
   constexpr int COLS = OUT_F32 ? 32 : 64;
-  if (CHECK_TAIL && (p.N & (VEC - 1)) != 0 && col + COLS > p.N) {
+  lim = min(lim, p.N);
+  if (CHECK_TAIL && col + COLS > lim && (lim < p.N || (p.N & (VEC - 1)) != 0)) {
     if (row < p.M) {
       if constexpr (OUT_F32) {
         float *dst = static_cast<float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
 #pragma unroll
         for (int j = 0; j < 32; ++j)
-          if (col + j < p.N) dst[j] = __uint_as_float(w[j]);
+          if (col + j < lim) dst[j] = __uint_as_float(w[j]);
       } else {
         __half *dst = static_cast<__half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
 #pragma unroll
         for (int j = 0; j < 32; ++j) {
           const __half2 hv = *reinterpret_cast<const __half2 *>(&w[j]);
-          if (col + 2 * j < p.N) dst[2 * j] = __low2half(hv);
-          if (col + 2 * j + 1 < p.N) dst[2 * j + 1] = __high2half(hv);
+          if (col + 2 * j < lim) dst[2 * j] = __low2half(hv);
+          if (col + 2 * j + 1 < lim) dst[2 * j + 1] = __high2half(hv);
         }
       }
     }
@@ -436,6 +446,12 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
   constexpr uint32_t B_HALF_BYTES = S::B_HALF_BYTES;
   constexpr uint32_t STAGE_BYTES = S::STAGE_BYTES;
   constexpr uint32_t IDESC = make_idesc_f16<BM * CG, UMMA_N, A_MN, B_MN, ACC16>();
+  // flexible tile width: TN columns per tile (NH == 1 only;
+  // the host sets it only for a K-major Bk, whole tiles, no stream-K / all-gather / multicast)
+  const int TN = (NH == 1 && MC == 1 && !AG && p.tile_n > 0) ? p.tile_n : BN;
+  const bool flex = TN != BN;
+  const int TB_ROWS = TN / CG;  // Bk rows per CTA per tile
+  const uint32_t idesc = flex ? ((IDESC & ~(0x3Fu << 17)) | (static_cast<uint32_t>(TN >> 3) << 17)) : IDESC;
   // FP16 accumulation (opt-in compute type, hgemm_ex): FP16 output, whole tiles only
   static_assert(!ACC16 || (!OUT_F32 && MC == 1 && !AG), "ACC16: FP16 out, no multicast / all-gather");
   // Per-K=16 advance of the descriptor start address (in bytes).
@@ -529,14 +545,15 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         // (alternating per item, so consecutive half items double-buffer TMEM)
         const bool half = (NH == 2) && (MC == 1) && sub >= 0;
         const int hsel = i & 1;
-        const uint32_t stage_bytes = half ? STAGE_BYTES - B_HALF_BYTES : STAGE_BYTES;
+        const uint32_t stage_bytes = half ? STAGE_BYTES - B_HALF_BYTES
+                                     : flex ? A_BYTES + static_cast<uint32_t>(TB_ROWS) * 128u : STAGE_BYTES;
         if (i == 0) {
           HG_STAMP2(1);
           griddep_wait();  // first global access of this role below
           HG_STAMP(2);
         }
         const int a_row = (tm * MC + static_cast<int>(pair)) * BM * CG + static_cast<int>(prank) * BM;
-        const int b_row0 = tn * BN + static_cast<int>(prank) * B_ROWS;
+        const int b_row0 = tn * TN + static_cast<int>(prank) * TB_ROWS;
         if constexpr (AG) {
           // fused all-gather: wait until every chunk of op(A) rows this tile reads
           // (tn*BN .. +BN) is complete in the local gather buffer
@@ -648,7 +665,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           const uint32_t b_addr = sa + A_BYTES + h * B_HALF_BYTES + k * B_KSTEP;
           const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
           const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
-          umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kbl | k) != 0 ? 1u : 0u);
+          umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, idesc, (kbl | k) != 0 ? 1u : 0u);
         }
       };
       WorkItem wi;
@@ -752,7 +769,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
                 for (int h = 0; h < NH; ++h) {
                   const uint32_t b_addr = sa + A_BYTES + h * B_HALF_BYTES + k * B_KSTEP;
                   const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
-                  umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, IDESC, (kb | k) != 0 ? 1u : 0u);
+                  umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, idesc, (kb | k) != 0 ? 1u : 0u);
                 }
               }
               umma_commit_mask<CG>(&empty[stage], empty_mask);
@@ -833,7 +850,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       const int nh_act = half ? 1 : NH;
       // D column of TMEM column 0 (a half item's data sits in TMEM half hsel but
       // belongs to D columns tn*BN + isub*UMMA_N ..)
-      const int cbase = tn * BN + (half ? (isub - hsel) * UMMA_N : 0);
+      const int cbase = tn * TN + (half ? (isub - hsel) * UMMA_N : 0);
+      const int tile_lim = cbase + TN;  // flexible tiles: the first column of the next tile
       // accumulator halves in visiting order: a half item hands its unused half back first
       auto half_at = [&](int hh) { return half ? (hh == 0 ? 1 - hsel : hsel) : hh; };
       // 0: whole tile; 1: a later k segment of a stream-K tile -> publish FP32
@@ -866,7 +884,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       // the rest are prefetched into L2 and loaded when their box is free.
       constexpr int NB = EPI_COLS_W / EPI_COLS;  // staging boxes per warp per accumulator half
       constexpr int NBT = NH * NB;               // ... per tile
-      const bool c_tma = beta != 0.0f && mode == 0 && (p.N & (VEC - 1)) == 0;
+      const bool c_tma = beta != 0.0f && mode == 0 && (p.N & (VEC - 1)) == 0 && !flex;
       const int nbt = nh_act * NB;               // boxes carrying data
       const uint32_t s0 = nstore;
       auto box_col = [&](int j) {
@@ -1084,16 +1102,22 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
 #pragma unroll
             for (int c = 0; c < RB; ++c) {
               uint32_t ns = 0;  // < EPI_BUFS: no buffer wait
-              emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, smem_u32(smem) + (ew * RB + c) * 4096u, ns,
-                                                       *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
-                                                       cbase + c0 + c * EPI_COLS, row, row_base, lane);
+              const int colc = cbase + c0 + c * EPI_COLS;
+              const uint32_t rs = smem_u32(smem) + (ew * RB + c) * 4096u;
+              const uint32_t(&wc)[32] = *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]);
+              if (!flex) emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, rs, ns, wc, colc, row, row_base, lane);
+              else if (colc < tile_lim)  // flexible tiles: stop at the tile end
+                emit_row_chunk<OUT_F32, EPI_BUFS, true>(p, &tmD, rs, ns, wc, colc, row, row_base, lane, tile_lim);
             }
           } else {
 #pragma unroll
-            for (int c = 0; c < RB; ++c)
-              emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, stg, nstore,
-                                                       *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]),
-                                                       cbase + c0 + c * EPI_COLS, row, row_base, lane);
+            for (int c = 0; c < RB; ++c) {
+              const int colc = cbase + c0 + c * EPI_COLS;
+              const uint32_t(&wc)[32] = *reinterpret_cast<const uint32_t(*)[32]>(&pk[c * 32]);
+              if (!flex) emit_row_chunk<OUT_F32, EPI_BUFS, false>(p, &tmD, stg, nstore, wc, colc, row, row_base, lane);
+              else if (colc < tile_lim)
+                emit_row_chunk<OUT_F32, EPI_BUFS, true>(p, &tmD, stg, nstore, wc, colc, row, row_base, lane, tile_lim);
+            }
           }
 #ifdef HGEMM_TRACE
           if (warp == 2 && lane == 0 && it == 0 && h == 0) HG_STAMP2(6);
@@ -1199,8 +1223,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             for (int j = 0; j < 32; ++j)
               w[j] = pack_half2(alpha * __uint_as_float(v[2 * j]), alpha * __uint_as_float(v[2 * j + 1]));
           }
+          if (col >= tile_lim) continue;  // flexible tiles: past the tile end (TMEM already released)
           if (beta != 0.0f && row < p.M) {
-            const int ncol = min(EPI_COLS, p.N - col);
+            const int ncol = min(EPI_COLS, min(p.N, tile_lim) - col);
             if constexpr (OUT_F32) {
               const float *src = static_cast<const float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
               if (ncol == 32) {
@@ -1243,7 +1268,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
               }
             }
           }
-          emit_row_chunk<OUT_F32, EPI_BUFS>(p, &tmD, stg, nstore, w, col, row, row_base, lane);
+          emit_row_chunk<OUT_F32, EPI_BUFS>(p, &tmD, stg, nstore, w, col, row, row_base, lane, tile_lim);
         }
       }
       if (warp == 2 && lane == 0) {

@@ -58,6 +58,12 @@ def test_set_config_validation():
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 256, 0, 0, 0, 2))) == 0
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 512, 0, 0, 0, 1, 2))) == 0   # half_tail 0..2
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 512, 0, 0, 0, 1, 3))) == 1
+    # flexible tile width: CTA pair, block_n 256, a multiple of 16 in [128, 256]
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 256, 0, 0, 0, 0, 0, 144))) == 0
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 256, 0, 0, 0, 0, 0, 136))) == 1
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 512, 0, 0, 0, 0, 0, 144))) == 1
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(2, 256, 0, 0, 0, 0, 0, 144))) == 1
+    assert lib.hgemm_set_config(ctypes.byref(binding._Config(3, 256, 0, 0, 0, 0, 0, 112))) == 1
     # HBM-streaming kernel: chunk width a multiple of 16 in [16, 256] (0 = auto)
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(5, 112, 0, 0))) == 0
     assert lib.hgemm_set_config(ctypes.byref(binding._Config(5, 0, 0, 0))) == 0

@@ -548,3 +548,38 @@ def test_stream_swapped_integer_exact(oracle_mod):
     assert case.stats["last_kernel"] == "stream" and case.stats["group_m"] == 1, case.stats
     _, r, _ = case.oracle(oracle_mod)
     assert np.array_equal(got.astype(np.float64), r)
+
+
+@pytest.mark.parametrize("tile_n", [128, 144, 160, 192, 240])
+@pytest.mark.parametrize("tA,tB", [("T", "N"), ("T", "T")])   # flexible widths need a K-major op(A)
+@pytest.mark.parametrize("out,beta", [("f16", 0.0), ("f32", 0.0), ("f16", 1.0), ("f32", -0.5)])
+def test_flexible_tile_width(oracle_mod, tile_n, tA, tB, out, beta):
+    """CTA-pair kernel with tiles of tile_n columns: chunks
+    that cross a tile end are stored directly, never by a TMA box running into the next tile."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("tc2", block_n=256, tile_n=tile_n)
+    m, n, k = 1000, 600, 328           # several tiles of every width + ragged m / n / k
+    C = inputs.uniform_f16(m, n, 23) if beta else None
+    case = GpuCase(inputs.uniform_f16(m, k, 21), inputs.uniform_f16(k, n, 22), tA, tB, beta=beta, C=C, out=out,
+                   pad=(8, 16, 8))
+    got = case.run_gpu()
+    assert case.stats["last_kernel"] == "tc2" and case.stats["tile_n"] == tile_n % 256, case.stats
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, got, r, ab)
+    assert np.all(np.isnan(case.padding(got).astype(np.float32)))
+    # integer inputs: bit-exact, and every element written exactly once (beta = 1 over an integer C)
+    opA = inputs.integer_f16(m, k, 24, -2, 2)
+    opB = inputs.integer_f16(k, n, 25, -2, 2)
+    Ci = inputs.integer_f16(m, n, 26, -4, 4)
+    case = GpuCase(opA, opB, tA, tB, beta=1.0, C=Ci, out="f32")
+    got = case.run_gpu()
+    _, r, _ = case.oracle(oracle_mod)
+    assert np.array_equal(case.view(got).astype(np.float64), r)
+
+
+@pytest.mark.parametrize("w", [1792, 2304, 2560])
+def test_flexible_tile_width_auto_mid_square(oracle_mod, w):
+    """The automatic choice at mid-size squares of the paper sweep, sampled against the oracle."""
+    from .test_gpu_large import _check_sampled
+    got, stats = _check_sampled(oracle_mod, w, w, w, "T", "N", 1.0, 0.0, "f16", seed=700)
+    assert stats["last_kernel"] in ("tc2", "tc1", "splitk"), stats

@@ -23,12 +23,15 @@ ap.add_argument("--warm", type=float, default=3.0)
 ap.add_argument("--iters", type=int, default=200)
 ap.add_argument("--order", default="ours,cublas,ours,cublas")
 ap.add_argument("--compute", default="f32", help="accumulation type of ours (f16: hgemm_ex FP16 accumulate)")
+ap.add_argument("--group-m", type=int, default=0, help="raster group height of ours (0 = library default)")
 args = ap.parse_args()
 m = n = k = args.m
 A = (torch.rand(m, k, device="cuda") * 2 - 1).half()    # op(A) rows, K-major: the paper's TN layout
 B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
 C = torch.empty(n, m, dtype=torch.half, device="cuda")
 torch.backends.cuda.matmul.allow_fp16_reduced_precision_reduction = False
+if args.group_m:
+    binding.set_config(group_m=args.group_m)
 
 
 def ours():

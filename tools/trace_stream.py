@@ -15,6 +15,10 @@ mb.mb_stamp.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
 st = torch.zeros(2, dtype=torch.int64, device="cuda")
 
 m, n, k = (int(x) for x in sys.argv[1:4]) if len(sys.argv) > 3 else (16384, 64, 4096)
+beta = float(sys.argv[4]) if len(sys.argv) > 4 else 0.0
+cw = int(sys.argv[5]) if len(sys.argv) > 5 else 0
+if "--force" in sys.argv or cw:
+    binding.set_config("stream", block_n=cw)
 A = (torch.rand(m, k, device="cuda") * 2 - 1).half()
 B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
 C = torch.empty(n, m, device="cuda", dtype=torch.half)
@@ -29,7 +33,7 @@ for i in range(6):
     if i == 5:
         e0.record()
         mb.mb_stamp(st.data_ptr(), torch.cuda.current_stream().cuda_stream)
-    binding.hgemm(m, n, k, 1.0, A, k, B, k, 0.0, C, m, "T", "N", "f16")
+    binding.hgemm(m, n, k, 1.0, A, k, B, k, beta, C, m, "T", "N", "f16")
     if i == 5:
         mb.mb_stamp(st.data_ptr() + 8, torch.cuda.current_stream().cuda_stream)
         e1.record()
@@ -40,7 +44,7 @@ v = probe.cpu().view(-1).tolist()
 rows = [v[8 * b: 8 * b + 8] for b in range(160) if v[8 * b]]
 t0 = min(x[0] for x in rows)
 names = ["start", "setup", "data0", "mma_done", "epi_wake", "epi_done", "end"]
-print(f"{len(rows)} CTAs; span {max(x[6] for x in rows) - t0} ns")
+print(f"{m}x{n}x{k} beta={beta}: {len(rows)} CTAs; span {max(x[6] for x in rows) - t0} ns")
 for f, nm in enumerate(names):
     xs = [x[f] - t0 for x in rows if x[f]]
     if xs:
