@@ -38,6 +38,8 @@ struct SkShape {
   static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr uint32_t PART_BYTES = BM * BN * 4;     // receive buffer: S x 128 rows x BN/S FP32
   static constexpr int STAGES_FIT = static_cast<int>((227u * 1024u - PART_BYTES - 2048u) / STAGE_BYTES);
+  // At most 6 stages: 8 for BN = 64 (every k-block of an LSTM-gate CTA in flight at once) fit
+  // but measured 0.9 us slower per launch (profiles/r02/splitk_stages_sweep.log)
   static constexpr int STAGES = STAGES_FIT > 6 ? 6 : STAGES_FIT;
   static constexpr uint32_t TMEM_COLS = BN < 32 ? 32 : BN;
   static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + PART_BYTES + 1024 + 1024;
