@@ -695,8 +695,12 @@ def run_ours(args, world, rank, local):
             Cc = C.clone()
             tc = timed(cublas_fn(A, Bs, Cc, tA, tB, alpha, beta), flush, args.warmup, args.steps, stream)
             diff = (Cc.float() - C.float()).abs().max().item() if beta == 0 else None
+            # tripwire: both accumulate in FP32, so they differ by ~1 output ulp at most
+            # (|C| <~ 6 sqrt(k/9) for uniform[-1,1) inputs); a larger difference is a bug
+            tol = 4.0 * 2.0 ** -10 * 6.0 * (k / 9.0) ** 0.5 if out == "f16" else 1e-4 * (k / 9.0) ** 0.5
             cublas = {"value": flops_rank / (tc["mean"] * 1e-3) / 1e12, "unit": UNIT, "ms": tc["mean"],
                       "ms_median": tc["median"], "max_abs_diff_vs_ours": diff,
+                      "agrees_with_ours": None if diff is None else bool(diff <= tol), "agree_tol": tol,
                       "what": ("torch.addmm(C, ..., beta, alpha, out=C)" if beta != 0 else "torch.mm") +
                               " (cuBLAS), same operands, layout and alpha/beta, fp16 reduced-precision reduction off,"
                               " same W warm-up and K flushed steps as ours"}

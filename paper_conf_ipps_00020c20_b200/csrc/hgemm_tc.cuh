@@ -450,7 +450,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
   // the host sets it only for a K-major Bk, whole tiles, no stream-K / all-gather / multicast)
   const int TN = (NH == 1 && MC == 1 && !AG && p.tile_n > 0) ? p.tile_n : BN;
   const bool flex = TN != BN;
-  const int TB_ROWS = TN / CG;  // Bk rows per CTA per tile
+  const int TB_ROWS = flex ? TN / CG : B_ROWS;  // Bk rows per CTA per tile (per accumulator half)
   const uint32_t idesc = flex ? ((IDESC & ~(0x3Fu << 17)) | (static_cast<uint32_t>(TN >> 3) << 17)) : IDESC;
   // FP16 accumulation (opt-in compute type, hgemm_ex): FP16 output, whole tiles only
   static_assert(!ACC16 || (!OUT_F32 && MC == 1 && !AG), "ACC16: FP16 out, no multicast / all-gather");
