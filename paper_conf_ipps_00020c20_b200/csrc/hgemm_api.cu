@@ -196,6 +196,11 @@ int sk_plan(int64_t tiles, int64_t units, int64_t nkb, int mode) {
 // Library-owned FP32 partial slots + flags, one set per (device, stream):
 // room for one 128 x 512 FP32 slot and one flag per SM.  Flags are zero
 // between launches (every consumer resets the flag it waited for).
+extern const int kWsyncOffset = 1024;  // ints: past the per-SM flags, on its own 128-B line
+extern const int g_env_wsync = [] {  // wave barrier: on unless HGEMM_WSYNC=0
+  const char *e = std::getenv("HGEMM_WSYNC");
+  return e ? std::atoi(e) : 1;
+}();
 struct SkWorkspace {
   int dev;
   cudaStream_t stream;
@@ -220,8 +225,9 @@ bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags)
   float *w = nullptr;
   int *f = nullptr;
   if (cudaMalloc(&w, static_cast<size_t>(num_sms) * 128 * 512 * sizeof(float)) != cudaSuccess) return false;
-  if (cudaMalloc(&f, static_cast<size_t>(num_sms) * sizeof(int)) != cudaSuccess ||
-      cudaMemsetAsync(f, 0, static_cast<size_t>(num_sms) * sizeof(int), s) != cudaSuccess) {
+  // flags: one per SM, then (at +kWsyncOffset ints) the wave-barrier counter
+  if (cudaMalloc(&f, static_cast<size_t>(kWsyncOffset + 32) * sizeof(int)) != cudaSuccess ||
+      cudaMemsetAsync(f, 0, static_cast<size_t>(kWsyncOffset + 32) * sizeof(int), s) != cudaSuccess) {
     cudaFree(w);
     if (f) cudaFree(f);
     return false;
@@ -721,6 +727,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   p.tile_n = tnf;
   p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
   p.group_m = cfg.group_m > 0 ? cfg.group_m : 16 / mc;  // measured best with 256x512 pair tiles (profiles/)
+
   p.group_m = std::max(1, std::min(p.group_m, p.num_m_tiles));
   if (g_env_group_n > 0)  // experiments: group along N instead
     p.group_m = -std::max(1, std::min(g_env_group_n, p.num_n_tiles));

@@ -31,8 +31,11 @@ extern thread_local bool t_half_used;     // the last tile launch of this thread
 
 // Stream-K plan (hgemm_api.cu): number of data-parallel tiles, or -1 for "no stream-K".
 int sk_plan(int64_t tiles, int64_t units, int64_t nkb, int mode);
-// Library-owned stream-K partial slots and flags for (device, stream) (hgemm_api.cu).
+// Library-owned stream-K partial slots and flags for (device, stream) (hgemm_api.cu);
+// flags + kWsyncOffset is the wave-barrier counter.
 bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags);
+extern const int kWsyncOffset;
+extern const int g_env_wsync;  // HGEMM_WSYNC: 1 = wave barrier for tile kernels with >= 8 whole waves
 
 // One launch of a persistent tile kernel.
 struct TcLaunch {
@@ -138,6 +141,23 @@ hgemm_status_t launch_tc(const TcLaunch &L) {
       p.sk_flags = flags;
       clusters = units;
       *L.sk_used = true;
+    }
+  }
+  // Wave barrier: with >= 8 whole waves of whole tiles, the
+  // producers of all CTAs meet before each wave, so the tiles that share Ak / Bk panels
+  // stream their k-blocks together instead of drifting apart over the waves (at 32768^3 the
+  // DRAM reads fall from 165 to 52 GB per launch).  Needs every cluster resident at once, as
+  // the grid is sized for (the stream-K fix-up relies on the same).  HGEMM_WSYNC=0 disables it.
+  p.wsync = nullptr;
+  p.wsync_items = 0;
+  if (g_env_wsync && MC == 1 && !AG && !*L.sk_used && clusters == units) {
+    const int whole_waves = (tiles - p.n_half) / units;
+    float *ws = nullptr;
+    int *flags = nullptr;
+    if (whole_waves >= 8 && units * CG <= di.num_sms && sk_workspace(dev, L.stream, di.num_sms, &ws, &flags) &&
+        cudaMemsetAsync(flags + kWsyncOffset, 0, sizeof(int), L.stream) == cudaSuccess) {
+      p.wsync = flags + kWsyncOffset;
+      p.wsync_items = whole_waves;
     }
   }
   cudaLaunchConfig_t cfg = {};

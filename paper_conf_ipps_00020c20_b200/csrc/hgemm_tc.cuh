@@ -87,6 +87,12 @@ struct TcParams {
   // tiles of tile_n columns (a multiple of 16, <= UMMA_N; 0 = BN), chosen by the host so the
   // tile count fills whole waves.
   int32_t tile_n;
+  // Wave barrier (experiment, HGEMM_WSYNC): before item i (0 < i < wsync_items) every CTA's
+  // producer waits until all CTAs' producers have issued their items < i, so the tiles of a
+  // wave start their k loops together and share their panels in L2.
+  // *wsync is zeroed by the host before the launch.
+  int *wsync;
+  int32_t wsync_items;
   int32_t exp_flags;  // experiments (HGEMM_EXP): 1 = no ring staging for the last item, 2 = no C-load hold-back,
                       // 4 = wait for store completion before exit, 8 = no PDL trigger, 16 = no cluster
                       // attribute for 1-CTA launches (host side)
@@ -551,6 +557,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           HG_STAMP2(1);
           griddep_wait();  // first global access of this role below
           HG_STAMP(2);
+        } else if (p.wsync != nullptr && i < p.wsync_items) {
+          atomicAdd(p.wsync, 1);  // this CTA has issued every load of its items < i
+          const int target = i * static_cast<int>(gridDim.x);
+          while (ld_acquire_gpu(p.wsync) < target) __nanosleep(64);
         }
         const int a_row = (tm * MC + static_cast<int>(pair)) * BM * CG + static_cast<int>(prank) * BM;
         const int b_row0 = tn * TN + static_cast<int>(prank) * TB_ROWS;

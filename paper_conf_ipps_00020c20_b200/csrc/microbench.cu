@@ -358,6 +358,29 @@ int mb_empty(int grid, int block, int smem, int cluster, unsigned long long *dst
   return cudaLaunchKernelEx(&cfg, empty_kernel, dst, smem > 0 ? 1 : 0) == cudaSuccess ? 0 : 1;
 }
 
+// cudaOccupancyMaxActiveClusters for a kernel of this launch shape (cluster size,
+// dynamic smem, block): how many clusters of that size the GPU holds at once.
+int mb_max_clusters(int cluster, int smem, int block) {
+  if (cudaFuncSetAttribute(empty_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448) != cudaSuccess)
+    return -2;
+  if (cluster > 8 && cudaFuncSetAttribute(empty_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess)
+    return -3;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(cluster * 64);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cudaLaunchAttribute a[1];
+  a[0].id = cudaLaunchAttributeClusterDimension;
+  a[0].val.clusterDim.x = cluster;
+  a[0].val.clusterDim.y = 1;
+  a[0].val.clusterDim.z = 1;
+  cfg.attrs = a;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, empty_kernel, &cfg) != cudaSuccess) return -1;
+  return n;
+}
+
 // One-thread kernel writing %globaltimer to *dst (timeline probes around a launch).
 int mb_stamp(unsigned long long *dst, cudaStream_t s) {
   stamp_kernel<<<1, 32, 0, s>>>(dst);
