@@ -201,6 +201,10 @@ extern const int g_env_wsync = [] {  // wave barrier: on unless HGEMM_WSYNC=0
   const char *e = std::getenv("HGEMM_WSYNC");
   return e ? std::atoi(e) : 1;
 }();
+extern const int g_env_wsync_k = [] {  // extra barriers every HGEMM_WSYNC_K k-blocks (-1 = automatic)
+  const char *e = std::getenv("HGEMM_WSYNC_K");
+  return e ? std::max(0, std::atoi(e)) : -1;
+}();
 struct SkWorkspace {
   int dev;
   cudaStream_t stream;

@@ -36,6 +36,7 @@ int sk_plan(int64_t tiles, int64_t units, int64_t nkb, int mode);
 bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags);
 extern const int kWsyncOffset;
 extern const int g_env_wsync;  // HGEMM_WSYNC: 1 = wave barrier for tile kernels with >= 8 whole waves
+extern const int g_env_wsync_k;  // HGEMM_WSYNC_K: k-block interval of extra barriers inside tiles (0 = none, -1 = auto)
 
 // One launch of a persistent tile kernel.
 struct TcLaunch {
@@ -143,21 +144,28 @@ hgemm_status_t launch_tc(const TcLaunch &L) {
       *L.sk_used = true;
     }
   }
-  // Wave barrier: with >= 8 whole waves of whole tiles, the
+  // Wave barrier: with >= 8 whole waves of whole tiles and K >= 8192, the
   // producers of all CTAs meet before each wave, so the tiles that share Ak / Bk panels
   // stream their k-blocks together instead of drifting apart over the waves (at 32768^3 the
   // DRAM reads fall from 165 to 52 GB per launch).  Needs every cluster resident at once, as
   // the grid is sized for (the stream-K fix-up relies on the same).  HGEMM_WSYNC=0 disables it.
   p.wsync = nullptr;
   p.wsync_items = 0;
+  p.wsync_kint = 0;
   if (g_env_wsync && MC == 1 && !AG && !*L.sk_used && clusters == units) {
     const int whole_waves = (tiles - p.n_half) / units;
     float *ws = nullptr;
     int *flags = nullptr;
-    if (whole_waves >= 8 && units * CG <= di.num_sms && sk_workspace(dev, L.stream, di.num_sms, &ws, &flags) &&
+    // long tiles only (K >= 8192): with short k loops the panels stay in L2 anyway and the
+    // per-wave meeting costs more than it saves (BERT-FFN1 16384 x 4096 x 1024: 129 -> 151 us)
+    if (whole_waves >= 8 && p.num_k_blocks >= 128 && units * CG <= di.num_sms &&
+        sk_workspace(dev, L.stream, di.num_sms, &ws, &flags) &&
         cudaMemsetAsync(flags + kWsyncOffset, 0, sizeof(int), L.stream) == cudaSuccess) {
       p.wsync = flags + kWsyncOffset;
       p.wsync_items = whole_waves;
+      // inside long tiles also every 64 k-blocks: at K >= 16384 the L2 read sectors fell by 16%
+      // and the sustained rate rose 1.5-3% (profiles/r02/wave_barrier_k_interval.log)
+      p.wsync_kint = g_env_wsync_k >= 0 ? g_env_wsync_k : (p.num_k_blocks >= 256 ? 64 : 0);
     }
   }
   cudaLaunchConfig_t cfg = {};

@@ -93,6 +93,7 @@ struct TcParams {
   // *wsync is zeroed by the host before the launch.
   int *wsync;
   int32_t wsync_items;
+  int32_t wsync_kint;  // > 0: also meet every wsync_kint k-blocks inside those tiles (experiment)
   int32_t exp_flags;  // experiments (HGEMM_EXP): 1 = no ring staging for the last item, 2 = no C-load hold-back,
                       // 4 = wait for store completion before exit, 8 = no PDL trigger, 16 = no cluster
                       // attribute for 1-CTA launches (host side)
@@ -543,6 +544,14 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       WorkItem wi;
       HG_STAMP2(0);
       bool cgo_sent = false;
+      // wave barrier (TcParams::wsync): every producer passes the same sequence of barrier
+      // points (wave starts, and every wsync_kint k-blocks inside the tiles of whole waves)
+      int nbar = 0;
+      auto wave_bar = [&]() {
+        atomicAdd(p.wsync, 1);
+        const int target = ++nbar * static_cast<int>(gridDim.x);
+        while (ld_acquire_gpu(p.wsync) < target) __nanosleep(64);
+      };
       for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i) {
         int tm, tn, tile, sub;
         item_tile(p, wi.tile, tile, sub);
@@ -558,9 +567,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           griddep_wait();  // first global access of this role below
           HG_STAMP(2);
         } else if (p.wsync != nullptr && i < p.wsync_items) {
-          atomicAdd(p.wsync, 1);  // this CTA has issued every load of its items < i
-          const int target = i * static_cast<int>(gridDim.x);
-          while (ld_acquire_gpu(p.wsync) < target) __nanosleep(64);
+          wave_bar();  // this CTA has issued every load of its items < i
         }
         const int a_row = (tm * MC + static_cast<int>(pair)) * BM * CG + static_cast<int>(prank) * BM;
         const int b_row0 = tn * TN + static_cast<int>(prank) * TB_ROWS;
@@ -578,6 +585,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           fence_proxy_async_global();  // the copy warps' generic stores -> this CTA's TMA (async proxy) reads
         }
         for (int kb = wi.kb0; kb < wi.kb1; ++kb) {
+          if (p.wsync_kint > 0 && p.wsync != nullptr && i < p.wsync_items && kb > wi.kb0 &&
+              (kb - wi.kb0) % p.wsync_kint == 0)
+            wave_bar();  // k-block alignment inside the tile (experiment, HGEMM_WSYNC_K)
           mbar_wait(&empty[stage], phase ^ 1u);
 #ifdef HGEMM_TRACE
           if (i == 0 && kb == wi.kb0) HG_STAMP2(2);
