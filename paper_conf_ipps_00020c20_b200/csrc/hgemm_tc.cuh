@@ -91,6 +91,7 @@ struct TcParams {
   // producer waits until all CTAs' producers have issued their items < i, so the tiles of a
   // wave start their k loops together and share their panels in L2.
   // *wsync is zeroed by the host before the launch.
+  int32_t l2_pf;  // > 0: the producer prefetches operand boxes this many k-blocks ahead into L2
   int *wsync;
   int32_t wsync_items;
   int32_t wsync_kint;  // > 0: also meet every wsync_kint k-blocks inside those tiles (experiment)
@@ -546,6 +547,30 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       bool cgo_sent = false;
       // wave barrier (TcParams::wsync): every producer passes the same sequence of barrier
       // points (wave starts, and every wsync_kint k-blocks inside the tiles of whole waves)
+      // L2 prefetch of k-block kbp's operand boxes (cp.async.bulk.prefetch.tensor): the ring's
+      // TMA loads then hit L2 instead of waiting for DRAM (the tiles of a wave march through k
+      // together, so every k-block is a fresh DRAM fetch)
+      auto l2_prefetch_kb = [&](int kbp, int a_row, int b_row0, bool half, int sub) {
+        const int kp = kbp * BK;
+        if constexpr (!A_MN) {
+          tma_prefetch_l2_2d(&tmA, kp, a_row);
+        } else {
+#pragma unroll
+          for (int q = 0; q < BM / 64; ++q) tma_prefetch_l2_2d(&tmA, a_row + 64 * q, kp);
+        }
+#pragma unroll
+        for (int hh = 0; hh < NH; ++hh) {
+          if (half && hh > 0) break;
+          const int b_row = b_row0 + (half ? sub : hh) * UMMA_N;
+          if constexpr (!B_MN) {
+            tma_prefetch_l2_2d(&tmB, kp, b_row);
+          } else {
+#pragma unroll
+            for (int q = 0; q < B_ROWS / 64; ++q) tma_prefetch_l2_2d(&tmB, b_row + 64 * q, kp);
+          }
+        }
+      };
+      int pf_next = 0;
       int nbar = 0;
       auto wave_bar = [&]() {
         atomicAdd(p.wsync, 1);
@@ -650,6 +675,11 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           if (i == 0 && kb == wi.kb0) HG_STAMP(3);
 #endif
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+          if (MC == 1 && p.l2_pf > 0) {  // keep the next l2_pf k-blocks of this tile prefetched into L2
+            if (kb == wi.kb0) pf_next = kb + 1;
+            const int pf_end = min(wi.kb1, kb + 1 + p.l2_pf);
+            for (; pf_next < pf_end; ++pf_next) l2_prefetch_kb(pf_next, a_row, b_row0, half, sub);
+          }
           // the first ring's worth of operand loads is queued: the epilogue's C loads
           // (beta != 0) may follow without delaying the start of the mainloop
           if (!cgo_sent && (i > 0 || kb + 1 - wi.kb0 >= STAGES || kb + 1 == wi.kb1)) {
