@@ -152,7 +152,9 @@ hgemm_status_t launch_tc(const TcLaunch &L) {
   p.wsync = nullptr;
   p.wsync_items = 0;
   p.wsync_kint = 0;
-  if (g_env_wsync && MC == 1 && !AG && !*L.sk_used && clusters == units) {
+  // (the fused all-gather kernel too: its copy warps never wait on a producer, so a producer
+  // held at the meeting cannot block the copies another producer is waiting for)
+  if (g_env_wsync && MC == 1 && !*L.sk_used && clusters == units) {
     const int whole_waves = (tiles - p.n_half) / units;
     float *ws = nullptr;
     int *flags = nullptr;

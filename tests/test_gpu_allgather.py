@@ -235,3 +235,9 @@ def test_two_processes_cuda_ipc(tmp_path):
     assert np.array_equal(cat, ref.cpu().numpy().view(np.uint16))
     for r in range(world):
         assert np.array_equal(np.load(os.path.join(tmp_path, f"gathered{r}.npy")), A.cpu().numpy().view(np.uint16))
+
+
+def test_fused_allgather_long_k_many_waves(oracle_mod):
+    """>= 8 whole waves and K >= 8192: the fused kernel runs with the wave barrier (DESIGN.md
+    "Wave barrier") while its copy warps pull the peer's rows; bitwise equal to hgemm()."""
+    _virtual(8192, 16384, 8192, 2, 4096, oracle_mod=oracle_mod)
