@@ -62,6 +62,7 @@ const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hi
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
 const bool g_env_flex = env_int("HGEMM_FLEX", 0) != 0;        // flexible tile widths in the automatic choice
 const int g_env_l2pf = env_int("HGEMM_L2PF", -1);             // L2 prefetch distance in k-blocks (-1 = automatic)
+const int g_env_direct = env_int("HGEMM_EPI_DIRECT", 0);      // 256-wide pair tiles: direct-store epilogue, 7 stages
 
 bool device_info(int dev, DeviceInfo &out) {
   if (dev < 0 || dev >= kMaxDevices) return false;
@@ -773,7 +774,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   const hgi::TcLaunch L = {&ta, &tb, &td, &p, dev, &di, cfg.max_ctas, skm_eff, &sk_used, stream};
   hgemm_status_t st;
   if (cg == 2 && bn == 512) st = hgi::dispatch_tc512(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
-  else if (cg == 2) st = hgi::dispatch_tc256x2(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
+  else if (cg == 2)
+    st = hgi::dispatch_tc256x2(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L, g_env_direct != 0 && !tnf);
   else st = hgi::dispatch_tc1(bn, a_mn, b_mn, f32, L);
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);

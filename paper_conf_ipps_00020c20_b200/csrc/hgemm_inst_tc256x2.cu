@@ -5,13 +5,22 @@
 
 namespace hgi {
 
-hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_mn, bool f32, const TcLaunch &L) {
+hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_mn, bool f32, const TcLaunch &L,
+                                bool direct) {
 #ifdef HGEMM_ENABLE_MC
   if (mc == 2) return dispatch_tc_layout<256, 2, 2>(a_mn, b_mn, f32, L);
 #endif
   (void)mc;
   if (ag) return dispatch_tc_ag<256>(a_mn, f32, L);
   if (acc16) return f32 ? HGEMM_ERR_INVALID_VALUE : dispatch_tc_acc16<256>(a_mn, b_mn, L);
+  // The direct-store epilogue variant (TcShape EPI_DIRECT: one more ring stage, 7 x 32 KB,
+  // instead of the staging boxes) measured slower on every shape (profiles/r02/
+  // epi_direct_experiment.log); it is instantiated only in experiment builds.
+#ifdef HGEMM_ENABLE_EPI_DIRECT
+  if (direct) return dispatch_tc_layout<256, 2, 1, true>(a_mn, b_mn, f32, L);
+#else
+  (void)direct;
+#endif
   return dispatch_tc_layout<256, 2, 1>(a_mn, b_mn, f32, L);
 }
 

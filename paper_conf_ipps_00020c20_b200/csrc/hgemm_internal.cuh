@@ -53,7 +53,8 @@ struct TcLaunch {
 // Per-family dispatchers (layout flags -> template instantiation), one per TU.
 //   acc16: FP16 accumulation (c_format = F16), FP16 output only, no all-gather / multicast.
 hgemm_status_t dispatch_tc512(int mc, bool ag, bool acc16, bool a_mn, bool b_mn, bool f32, const TcLaunch &L);
-hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_mn, bool f32, const TcLaunch &L);
+hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_mn, bool f32, const TcLaunch &L,
+                                bool direct = false);
 hgemm_status_t dispatch_tc1(int bn, bool a_mn, bool b_mn, bool f32, const TcLaunch &L);
 hgemm_status_t dispatch_splitk64(int spl, bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta,
                                  const CUtensorMap &tb, const hg::TcParams &p, int dev, cudaStream_t s);
@@ -70,16 +71,16 @@ struct KernInit {
   int max_clusters[kMaxDevices] = {};
 };
 
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC, bool AG, bool ACC16>
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC, bool AG, bool ACC16, bool DIRECT = false>
 hgemm_status_t launch_tc(const TcLaunch &L) {
-  using S = hg::TcShape<BN, CG, OUT_F32>;
+  using S = hg::TcShape<BN, CG, OUT_F32, DIRECT>;
   constexpr int THREADS = S::THREADS + (AG ? 32 : 0);  // + the all-gather copy warp
   const int dev = L.dev;
   const DeviceInfo &di = *L.di;
   const hg::TcParams &p0 = *L.p;
   const int ht_mode = L.sk_mode >> 4;  // hgemm_config_t::half_tail, packed above the stream-K mode
   const int sk_mode = L.sk_mode & 15;
-  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC, AG, ACC16>;
+  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC, AG, ACC16, DIRECT>;
   static KernInit init;
   std::call_once(init.once[dev], [&] {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, S::SMEM_BYTES);
@@ -195,10 +196,10 @@ hgemm_status_t launch_tc(const TcLaunch &L) {
 }
 
 // All eight (op(B) MN-major, op(A) MN-major, FP32 out) combinations of one tile shape.
-template <int BN, int CG, int MC>
+template <int BN, int CG, int MC, bool DIRECT = false>
 hgemm_status_t dispatch_tc_layout(bool a_mn, bool b_mn, bool f32, const TcLaunch &L) {
 #define HG_CASE(AM, BM_, F) \
-  if (a_mn == AM && b_mn == BM_ && f32 == F) return launch_tc<BN, CG, AM, BM_, F, MC, false, false>(L);
+  if (a_mn == AM && b_mn == BM_ && f32 == F) return launch_tc<BN, CG, AM, BM_, F, MC, false, false, DIRECT>(L);
   HG_CASE(false, false, false)
   HG_CASE(false, false, true)
   HG_CASE(false, true, false)

@@ -237,7 +237,7 @@ __device__ __forceinline__ uint32_t pack_half2(float a, float b) {
   return *reinterpret_cast<uint32_t *>(&h);
 }
 
-template <int BN, int CG, bool OUT_F32>
+template <int BN, int CG, bool OUT_F32, bool EPI_DIRECT = false>
 struct TcShape {
   static constexpr int BM = 128;                       // rows per CTA (TMEM lanes)
   static constexpr int BK = 64;                        // FP16 per 128-B swizzle atom
@@ -258,10 +258,12 @@ struct TcShape {
   // beta = 1 and 256-wide tiles: 5 -> 6 stages, +6%).
   static constexpr int EPI_WARPS = 8;
   static constexpr int EPI_COLS_W = UMMA_N / 2;        // columns per warp per accumulator half
+  // EPI_DIRECT: no staging boxes -- the epilogue stores from registers, and the 32 KB go to
+  // one more ring stage
 #ifdef HGEMM_EPI_BUFS
-  static constexpr int EPI_BUFS = HGEMM_EPI_BUFS;
+  static constexpr int EPI_BUFS = EPI_DIRECT ? 0 : HGEMM_EPI_BUFS;
 #else
-  static constexpr int EPI_BUFS = 1;
+  static constexpr int EPI_BUFS = EPI_DIRECT ? 0 : 1;
 #endif
   static constexpr uint32_t EPI_BYTES = EPI_WARPS * EPI_BUFS * 32 * 128;
   // As many ring stages as fit in 227 KB next to the staging buffers, barriers and alignment slack.
@@ -288,6 +290,31 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
   constexpr int VEC = OUT_F32 ? 4 : 8;
   constexpr int COLS = OUT_F32 ? 32 : 64;
   lim = min(lim, p.N);
+  if constexpr (EPI_BUFS == 0) {  // direct-store epilogue: 16-B stores of the thread's row, masked at lim
+    if (row < p.M) {
+      if (col + COLS <= lim) {
+        uint4 *dst = reinterpret_cast<uint4 *>(static_cast<char *>(p.D) +
+                                               (static_cast<int64_t>(row) * p.ldd + col) * (OUT_F32 ? 4 : 2));
+#pragma unroll
+        for (int q = 0; q < 8; ++q) dst[q] = make_uint4(w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
+      } else if constexpr (OUT_F32) {
+        float *dst = static_cast<float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+#pragma unroll
+        for (int j = 0; j < 32; ++j)
+          if (col + j < lim) dst[j] = __uint_as_float(w[j]);
+      } else {
+        __half *dst = static_cast<__half *>(p.D) + static_cast<int64_t>(row) * p.ldd + col;
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const __half2 hv = *reinterpret_cast<const __half2 *>(&w[j]);
+          if (col + 2 * j < lim) dst[2 * j] = __low2half(hv);
+          if (col + 2 * j + 1 < lim) dst[2 * j + 1] = __high2half(hv);
+        }
+      }
+    }
+    (void)tmD; (void)stg; (void)nstore; (void)row_base; (void)lane;
+    return;
+  } else
   if (CHECK_TAIL && col + COLS > lim && (lim < p.N || (p.N & (VEC - 1)) != 0)) {
     if (row < p.M) {
       if constexpr (OUT_F32) {
@@ -308,9 +335,9 @@ __device__ __forceinline__ void emit_row_chunk(const TcParams &p, const CUtensor
     return;
   }
   // stage the 32 x 128-B box (SWIZZLE_128B: 16-B chunk q of row r at q ^ (r % 8))
-  const uint32_t sbuf = stg + (nstore % EPI_BUFS) * (32u * 128u);
+  const uint32_t sbuf = stg + (nstore % (EPI_BUFS > 0 ? EPI_BUFS : 1)) * (32u * 128u);
   if (nstore >= EPI_BUFS) {
-    if (lane == 0) bulk_wait_group_read<EPI_BUFS - 1>();  // the store that used this buffer has read it
+    if (lane == 0) bulk_wait_group_read<(EPI_BUFS > 0 ? EPI_BUFS : 1) - 1>();  // the store that used this buffer has read it
     __syncwarp();
   }
   const uint32_t rowaddr = sbuf + lane * 128u;
@@ -434,12 +461,13 @@ __device__ __forceinline__ void ag_copy_warp(const TcParams &p, uint32_t lane) {
   }
 }
 
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC = 1, bool AG = false, bool ACC16 = false>
-__global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 : 0), 1)
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC = 1, bool AG = false, bool ACC16 = false,
+          bool EPI_DIRECT = false>
+__global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS + (AG ? 32 : 0), 1)
     hgemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmD, const TcParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
-  using S = TcShape<BN, CG, OUT_F32>;
+  using S = TcShape<BN, CG, OUT_F32, EPI_DIRECT>;
   constexpr int BM = S::BM;
   constexpr int BK = S::BK;
   constexpr int UMMA_N = S::UMMA_N;
@@ -934,7 +962,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
       // the rest are prefetched into L2 and loaded when their box is free.
       constexpr int NB = EPI_COLS_W / EPI_COLS;  // staging boxes per warp per accumulator half
       constexpr int NBT = NH * NB;               // ... per tile
-      const bool c_tma = beta != 0.0f && mode == 0 && (p.N & (VEC - 1)) == 0 && !flex;
+      const bool c_tma = beta != 0.0f && mode == 0 && (p.N & (VEC - 1)) == 0 && !flex && EPI_BUFS > 0;
       const int nbt = nh_act * NB;               // boxes carrying data
       const uint32_t s0 = nstore;
       auto box_col = [&](int j) {
@@ -942,7 +970,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
                     : tn * BN + (j / NB) * UMMA_N + cgrp * EPI_COLS_W + (j % NB) * EPI_COLS;
       };
       auto c_load = [&](int j) {
-        const uint32_t b = (s0 + static_cast<uint32_t>(j)) % EPI_BUFS;
+        const uint32_t b = (s0 + static_cast<uint32_t>(j)) % (EPI_BUFS > 0 ? EPI_BUFS : 1);
         mbar_arrive_expect_tx(&skbar[ew * 2 + b], 32u * 128u);
         tma_load_2d(&tmD, stg + b * (32u * 128u), smem_u32(&skbar[ew * 2 + b]), box_col(j), row_base, 0);
       };
@@ -1035,7 +1063,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
               }
             }
             const bool in_ring = ring_c && j >= EPI_BUFS;
-            const uint32_t b = (s0 + static_cast<uint32_t>(j)) % EPI_BUFS;
+            const uint32_t b = (s0 + static_cast<uint32_t>(j)) % (EPI_BUFS > 0 ? EPI_BUFS : 1);
             uint32_t sbuf;
             if (in_ring) {
               mbar_wait(&skbar[ew * 2 + 1], 0u);  // single use per launch
@@ -1148,7 +1176,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
           // in its own ring slot instead of waiting for the staging buffer to be read.
           constexpr int RB = EPI_COLS_W / EPI_COLS;  // boxes per warp per accumulator half
           static_assert(S::EPI_WARPS * RB * 4096u <= STAGES * STAGE_BYTES, "ring staging");
-          if (last_item && p.sk_units == 0 && hh == NH - 1 && !(p.exp_flags & 1)) {
+          if (EPI_BUFS > 0 && last_item && p.sk_units == 0 && hh == NH - 1 && !(p.exp_flags & 1)) {
 #pragma unroll
             for (int c = 0; c < RB; ++c) {
               uint32_t ns = 0;  // < EPI_BUFS: no buffer wait
@@ -1212,11 +1240,22 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
             }
           }
           if (mode == 1) {  // publish this chunk of the partial accumulator: 4-KB boxes, bulk stores
+            if constexpr (EPI_BUFS == 0) {  // direct-store epilogue: the same swizzled boxes, 16-B stores
+#pragma unroll
+              for (int x = 0; x < EPI_COLS / 32; ++x) {
+                uint8_t *box = sk_box(cluster_id, (h * NCH + c) * (EPI_COLS / 32) + x) + lane * 128u;
+#pragma unroll
+                for (int q = 0; q < 8; ++q)
+                  *reinterpret_cast<uint4 *>(box + ((q ^ (lane & 7u)) << 4)) =
+                      make_uint4(v[32 * x + 4 * q], v[32 * x + 4 * q + 1], v[32 * x + 4 * q + 2], v[32 * x + 4 * q + 3]);
+              }
+              continue;
+            }
 #pragma unroll
             for (int x = 0; x < EPI_COLS / 32; ++x) {
-              const uint32_t sbuf = stg + (nstore % EPI_BUFS) * (32u * 128u);
+              const uint32_t sbuf = stg + (nstore % (EPI_BUFS > 0 ? EPI_BUFS : 1)) * (32u * 128u);
               if (nstore >= EPI_BUFS) {
-                if (lane == 0) bulk_wait_group_read<EPI_BUFS - 1>();
+                if (lane == 0) bulk_wait_group_read<(EPI_BUFS > 0 ? EPI_BUFS : 1) - 1>();
                 __syncwarp();
               }
               const uint32_t rowaddr = sbuf + lane * 128u;
@@ -1326,6 +1365,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32>::THREADS + (AG ? 32 :
         HG_CTRACE(it, 2);
       }
       if (mode == 1) {  // every epilogue warp's bulk stores of the slot have completed
+        if constexpr (EPI_BUFS == 0) {  // direct stores: visible to the head's bulk (async-proxy) loads
+          fence_proxy_async_global();
+          __threadfence();
+        }
         if (lane == 0) {
           bulk_wait_group<0>();
           fence_proxy_async_global();
