@@ -42,8 +42,19 @@
  * the same semantics (never an error; n > 65535*64 runs as several launches
  * over column ranges).  All indexing is 64-bit.
  *
- * Thread safety: hgemm() is reentrant; per-device properties are cached.
+ * Thread safety: hgemm() is reentrant; per-device properties and per-kernel
+ * launch setup are cached (initialised once per device, std::call_once).
  * hgemm_set_config() is process-global and meant for tests and benchmarks.
+ *
+ * Co-residency: the persistent tile kernels size their grid to the clusters
+ * the GPU holds at once.  Two features make CTAs of one launch wait for each
+ * other and so assume that all of them become resident: the stream-K fix-up
+ * (heads wait for the partials of later clusters) and the wave barrier
+ * (launches with >= 8 whole waves and K >= 8192: the producers meet before
+ * each wave).  On a GPU shared with other work a not-yet-resident cluster
+ * only delays the others; under MPS / green contexts with fewer SMs than
+ * the device reports, disable them (hgemm_config_t.stream_k = 1, environment
+ * HGEMM_WSYNC=0).
  */
 #ifndef HGEMM_H_
 #define HGEMM_H_

@@ -296,7 +296,37 @@ __global__ void teardown_kernel(int mode, uint8_t *gdst) {
 #endif
 }
 
+// Placement probe: every CTA of a cluster launch (the GEMM's shape) records %smid.
+__global__ void smid_kernel(int *out) {
+  extern __shared__ uint8_t sm[];
+  if (threadIdx.x == 0) {
+    uint32_t id;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(id));
+    out[blockIdx.x] = static_cast<int>(id);
+    sm[0] = 1;
+  }
+}
+
 extern "C" {
+
+// out[b] = %smid of CTA b for a grid of `grid` CTAs in clusters of `cluster` with `smem` bytes.
+int mb_smid(int grid, int cluster, int smem, int *out, cudaStream_t s) {
+  if (cudaFuncSetAttribute(smid_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448) != cudaSuccess)
+    return 2;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(128);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute a[1];
+  a[0].id = cudaLaunchAttributeClusterDimension;
+  a[0].val.clusterDim.x = cluster;
+  a[0].val.clusterDim.y = 1;
+  a[0].val.clusterDim.z = 1;
+  cfg.attrs = a;
+  cfg.numAttrs = cluster > 0 ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, smid_kernel, out) == cudaSuccess ? 0 : 1;
+}
 
 int mb_teardown(int grid, int block, int smem, int cluster, int mode, int pdl, void *gdst, cudaStream_t s) {
   static int attr = 0;
