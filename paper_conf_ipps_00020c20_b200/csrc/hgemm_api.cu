@@ -970,9 +970,16 @@ hgemm_status_t hgemm_host(int64_t m, int64_t n, int64_t k, float alpha, const vo
   }
   for (int64_t j = 1; j < panels; ++j) {
     const int64_t n0 = j * pw, n1 = std::min(n, n0 + pw);
-    if (!copy_b(n0, n1)) return fail(HGEMM_ERR_CUDA);
-    const hgemm_status_t st = gemm_step(0, m, n0, n1);
-    if (st != HGEMM_SUCCESS) return fail(st);
+    // the last panel goes in up to 4 slices (>= 256 columns each): only the last slice's GEMM
+    // and device->host copy remain after the final host->device copy (the pipeline's tail)
+    const int64_t slices = (j == panels - 1 && panels > 1) ? std::max<int64_t>(1, std::min<int64_t>(4, (n1 - n0) / 256)) : 1;
+    const int64_t sw = align_up(cdiv(n1 - n0, slices), 8);
+    for (int64_t s0 = n0; s0 < n1; s0 += sw) {
+      const int64_t s1 = std::min(n1, s0 + sw);
+      if (!copy_b(s0, s1)) return fail(HGEMM_ERR_CUDA);
+      const hgemm_status_t st = gemm_step(0, m, s0, s1);
+      if (st != HGEMM_SUCCESS) return fail(st);
+    }
   }
   // make `stream` observe the end of the pipeline (events recorded on it bracket the whole call)
   if (cudaEventRecord(P.ev_comp[HostPipe::kEv - 1], P.s_out) != cudaSuccess) return fail(HGEMM_ERR_CUDA);

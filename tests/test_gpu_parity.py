@@ -394,6 +394,25 @@ def test_hgemm_host_buffers(oracle_mod, tA, tB, out, beta):
     assert np.all(np.isnan(pad))
 
 
+@pytest.mark.parametrize("tA,tB", [("T", "N"), ("N", "T")])
+def test_hgemm_host_row_pieces(oracle_mod, tA, tB):
+    """m >= 4096: the first column panel's GEMM runs in row pieces of op(A) (started as their
+    rows arrive), the last panel in slices; beta = 1 so every element is written exactly once."""
+    import torch
+    from paper_conf_ipps_00020c20_b200 import binding
+    m, n, k = 4100, 2600, 264
+    case = GpuCase(inputs.integer_f16(m, k, 61, -2, 2), inputs.integer_f16(k, n, 62, -2, 2), tA, tB, 1.0, 1.0,
+                   C=inputs.integer_f16(m, n, 63, -4, 4), out="f32", pad=(3, 5, 7), align=False)
+    hA = torch.from_numpy(case.A.view(np.int16).copy()).pin_memory()
+    hB = torch.from_numpy(case.B.view(np.int16).copy()).pin_memory()
+    hC = torch.from_numpy(case.C_in.copy()).pin_memory()
+    ws = torch.empty(binding.host_workspace_size(m, n, k, tA, tB, "f32"), dtype=torch.uint8, device="cuda")
+    binding.hgemm_host(m, n, k, 1.0, hA, case.lda, hB, case.ldb, 1.0, hC, case.ldc, tA, tB, "f32", ws)
+    _, r, _ = case.oracle(oracle_mod)
+    assert np.array_equal(case.view(hC.numpy()).astype(np.float64), r)
+    assert np.all(np.isnan(case.padding(hC.numpy())))
+
+
 # ------------------------------------------------------------------ HBM-streaming kernel (skinny, TN)
 @pytest.mark.parametrize("n", [64, 100, 128, 200, 256])
 @pytest.mark.parametrize("cw,max_ctas", [(48, 0), (112, 3), (16, 5), (128, 0)])
