@@ -422,7 +422,7 @@ def strong_32768(args, world, rank, dev, flush, steps=5, warmup=2):
     problem alone (t1) so the record carries t1 / (N * t_gemm)."""
     import torch
     from paper_conf_ipps_00020c20_b200 import binding
-    from paper_conf_ipps_00020c20_b200.sharded import broadcast_A, hgemm_sharded, slab_bounds
+    from paper_conf_ipps_00020c20_b200.sharded import slab_bounds
     m = n = k = 32768
     n0, n1 = slab_bounds(n, world, rank)
     ns = n1 - n0

@@ -641,10 +641,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
           if (p.wsync_kint > 0 && p.wsync != nullptr && i < p.wsync_items && kb > wi.kb0 &&
               (kb - wi.kb0) % p.wsync_kint == 0)
             wave_bar();  // k-block alignment inside the tile (experiment, HGEMM_WSYNC_K)
-          // the producer runs ahead of the MMAs: a hardware-suspended wait (try_wait with a
-          // time hint) instead of a polling loop; HGEMM_EXP & 64 polls
-          if (p.exp_flags & 64) mbar_wait(&empty[stage], phase ^ 1u);
-          else mbar_wait_sleep(&empty[stage], phase ^ 1u);
+          // polling: a hardware-suspended wait (try_wait with a time hint, HGEMM_EXP & 64) wakes
+          // up late and measured slower on every mid-size shape
+          if (p.exp_flags & 64) mbar_wait_sleep(&empty[stage], phase ^ 1u);
+          else mbar_wait(&empty[stage], phase ^ 1u);
 #ifdef HGEMM_TRACE
           if (i == 0 && kb == wi.kb0) HG_STAMP2(2);
 #endif
@@ -990,8 +990,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
       // One thread polls the accumulator barrier; the other epilogue warps
       // sleep on a named barrier instead of spinning.
       if (warp == 2 && lane == 0) {
-        if (p.exp_flags & 64) mbar_wait(&tfull[buf * NH], acc_phase);
-        else mbar_wait_sleep(&tfull[buf * NH], acc_phase);  // the whole mainloop long: suspended, not polling
+        if (p.exp_flags & 64) mbar_wait_sleep(&tfull[buf * NH], acc_phase);  // experiment
+        else mbar_wait(&tfull[buf * NH], acc_phase);
         HG_TRACE(it, 1);
         for (int c2 = cluster_id + 1; c2 < c_hi; ++c2) {  // mode 2: wait for the published partials
           int *f = p.sk_flags + c2 * CG + static_cast<int>(rank);
@@ -1035,7 +1035,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
         for (int hh = 0; hh < NH; ++hh) {
           const int h = half_at(hh);
           if (h > 0) {
-            if (lane == 0) mbar_wait_sleep(&tfull[buf * NH + h], acc_phase);
+            if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
             __syncwarp();
             tc_fence_after();
           }
@@ -1122,7 +1122,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
         for (int hh = 0; hh < NH; ++hh) {
           const int h = half_at(hh);
           if (h > 0) {  // each half has its own tmem_full barrier
-            if (lane == 0) mbar_wait_sleep(&tfull[buf * NH + h], acc_phase);
+            if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
             __syncwarp();
             tc_fence_after();
           }
@@ -1211,7 +1211,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
       for (int hh = 0; hh < NH; ++hh) {
         const int h = half_at(hh);
         if (h > 0) {
-          if (lane == 0) mbar_wait_sleep(&tfull[buf * NH + h], acc_phase);
+          if (lane == 0) mbar_wait(&tfull[buf * NH + h], acc_phase);
           __syncwarp();
           tc_fence_after();
         }
