@@ -61,7 +61,6 @@ const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster gro
 const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hints
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
 const bool g_env_flex = env_int("HGEMM_FLEX", 0) != 0;        // flexible tile widths in the automatic choice
-const int g_env_l2pf = env_int("HGEMM_L2PF", -1);             // L2 prefetch distance in k-blocks (-1 = automatic)
 const int g_env_direct = env_int("HGEMM_EPI_DIRECT", 0);      // 256-wide pair tiles: direct-store epilogue, 7 stages
 
 bool device_info(int dev, DeviceInfo &out) {
@@ -567,7 +566,6 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
                                                        (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
     p.probe = g_probe.load(std::memory_order_relaxed);
     p.k_rot = g_env_stream_rot;
-    p.l2_pf = g_env_l2pf >= 0 ? g_env_l2pf : 0;
     p.alpha = alpha;
     p.beta = beta;
     p.D = C;
@@ -616,7 +614,6 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
                                                        (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
     p.probe = g_probe.load(std::memory_order_relaxed);
     p.k_rot = 1;
-    p.l2_pf = g_env_l2pf >= 0 ? g_env_l2pf : 0;
     p.alpha = alpha;
     p.beta = beta;
     p.D = C;
@@ -667,7 +664,6 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
       p.num_n_tiles = static_cast<int32_t>(cdiv(N, sk_bn));
       p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
       p.group_m = p.num_m_tiles;  // tiles in m-fastest order
-      p.l2_pf = g_env_l2pf >= 0 ? g_env_l2pf : 0;
       p.alpha = alpha;
       p.beta = beta;
       p.D = C;
@@ -741,7 +737,6 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   if (g_env_group_n > 0)  // experiments: group along N instead
     p.group_m = -std::max(1, std::min(g_env_group_n, p.num_n_tiles));
   p.l2_hint = g_env_l2_hint;
-  p.l2_pf = g_env_l2pf >= 0 ? g_env_l2pf : 0;
   p.exp_flags = g_env_exp;
   if (ag) {
     p.ag_ctr = ag->ctr;

@@ -169,15 +169,6 @@ __global__ void __launch_bounds__(192, 1)
     }
     fence_mbarrier_init();
     griddep_wait();
-    if (p.l2_pf > 0)  // the rest of this CTA's k range into L2 at once (one HBM round trip)
-      for (int kb = kb0 + STAGES; kb < kb1; ++kb) {
-        if constexpr (!A_MN) tma_prefetch_l2_2d(&tmA, kb * BK, a_row);
-        else
-          for (int q = 0; q < BM / 64; ++q) tma_prefetch_l2_2d(&tmA, a_row + 64 * q, kb * BK);
-        if constexpr (!B_MN) tma_prefetch_l2_2d(&tmB, kb * BK, b_row);
-        else
-          for (int q = 0; q < BN / 64; ++q) tma_prefetch_l2_2d(&tmB, b_row + 64 * q, kb * BK);
-      }
     produce(min(kb1, kb0 + STAGES));
   }
   if (warp == 1) {

@@ -50,7 +50,6 @@ struct StreamParams {
   // resident, computing C = op(A) op(B) with C column-major; each warp's 32 rows
   // are consecutive in memory, so every column store is one 64/128-B segment)
   int32_t tout;
-  int32_t l2_pf;  // > 0: prefetch the streamed operand's boxes this many k-blocks ahead into L2
 };
 
 #ifdef HGEMM_TRACE
@@ -126,8 +125,6 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll
       for (int t = 0; t < MT; ++t) tma_load_2d(&tmA, sa + t * A_SUB, fb, kb * 64, t * 128, 0);
       tma_load_2d(&tmB, sa + a_bytes, fb, kb * 64, pch * cw, 0);
-      if (p.l2_pf > 0 && pi + p.l2_pf < nkb)  // more HBM requests in flight than the smem ring holds
-        tma_prefetch_l2_2d(&tmB, ((pi + p.l2_pf + kb_rot) % nkb) * 64, pch * cw);
       if (++pstage == static_cast<uint32_t>(stages)) { pstage = 0; pphase ^= 1u; }
       if (++pi == nkb) { pi = 0; pch += gridDim.x; }
     }
@@ -144,9 +141,6 @@ __global__ void __launch_bounds__(192, 1)
     }
     fence_mbarrier_init();
     griddep_wait();
-    if (p.l2_pf > 0 && blockIdx.x < p.num_chunks)  // the first chunk's k-blocks beyond the first ring
-      for (int q = stages; q < min(nkb, stages + p.l2_pf); ++q)
-        tma_prefetch_l2_2d(&tmB, ((q + kb_rot) % nkb) * 64, static_cast<int>(blockIdx.x) * cw);
     produce(stages);
   }
   if (warp == 1) {

@@ -91,7 +91,6 @@ struct TcParams {
   // producer waits until all CTAs' producers have issued their items < i, so the tiles of a
   // wave start their k loops together and share their panels in L2.
   // *wsync is zeroed by the host before the launch.
-  int32_t l2_pf;  // > 0: the producer prefetches operand boxes this many k-blocks ahead into L2
   int *wsync;
   int32_t wsync_items;
   int32_t wsync_kint;  // > 0: also meet every wsync_kint k-blocks inside those tiles (experiment)
@@ -575,30 +574,6 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
       bool cgo_sent = false;
       // wave barrier (TcParams::wsync): every producer passes the same sequence of barrier
       // points (wave starts, and every wsync_kint k-blocks inside the tiles of whole waves)
-      // L2 prefetch of k-block kbp's operand boxes (cp.async.bulk.prefetch.tensor): the ring's
-      // TMA loads then hit L2 instead of waiting for DRAM (the tiles of a wave march through k
-      // together, so every k-block is a fresh DRAM fetch)
-      auto l2_prefetch_kb = [&](int kbp, int a_row, int b_row0, bool half, int sub) {
-        const int kp = kbp * BK;
-        if constexpr (!A_MN) {
-          tma_prefetch_l2_2d(&tmA, kp, a_row);
-        } else {
-#pragma unroll
-          for (int q = 0; q < BM / 64; ++q) tma_prefetch_l2_2d(&tmA, a_row + 64 * q, kp);
-        }
-#pragma unroll
-        for (int hh = 0; hh < NH; ++hh) {
-          if (half && hh > 0) break;
-          const int b_row = b_row0 + (half ? sub : hh) * UMMA_N;
-          if constexpr (!B_MN) {
-            tma_prefetch_l2_2d(&tmB, kp, b_row);
-          } else {
-#pragma unroll
-            for (int q = 0; q < B_ROWS / 64; ++q) tma_prefetch_l2_2d(&tmB, b_row + 64 * q, kp);
-          }
-        }
-      };
-      int pf_next = 0;
       int nbar = 0;
       auto wave_bar = [&]() {
         atomicAdd(p.wsync, 1);
@@ -641,10 +616,9 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
           if (p.wsync_kint > 0 && p.wsync != nullptr && i < p.wsync_items && kb > wi.kb0 &&
               (kb - wi.kb0) % p.wsync_kint == 0)
             wave_bar();  // k-block alignment inside the tile (experiment, HGEMM_WSYNC_K)
-          // polling: a hardware-suspended wait (try_wait with a time hint, HGEMM_EXP & 64) wakes
-          // up late and measured slower on every mid-size shape
-          if (p.exp_flags & 64) mbar_wait_sleep(&empty[stage], phase ^ 1u);
-          else mbar_wait(&empty[stage], phase ^ 1u);
+          // polling: a hardware-suspended wait (try_wait with a time hint) woke up late and
+          // measured slower on every mid-size shape
+          mbar_wait(&empty[stage], phase ^ 1u);
 #ifdef HGEMM_TRACE
           if (i == 0 && kb == wi.kb0) HG_STAMP2(2);
 #endif
@@ -706,11 +680,6 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
           if (i == 0 && kb == wi.kb0) HG_STAMP(3);
 #endif
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
-          if (MC == 1 && p.l2_pf > 0) {  // keep the next l2_pf k-blocks of this tile prefetched into L2
-            if (kb == wi.kb0) pf_next = kb + 1;
-            const int pf_end = min(wi.kb1, kb + 1 + p.l2_pf);
-            for (; pf_next < pf_end; ++pf_next) l2_prefetch_kb(pf_next, a_row, b_row0, half, sub);
-          }
           // the first ring's worth of operand loads is queued: the epilogue's C loads
           // (beta != 0) may follow without delaying the start of the mainloop
           if (!cgo_sent && (i > 0 || kb + 1 - wi.kb0 >= STAGES || kb + 1 == wi.kb1)) {
@@ -990,8 +959,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
       // One thread polls the accumulator barrier; the other epilogue warps
       // sleep on a named barrier instead of spinning.
       if (warp == 2 && lane == 0) {
-        if (p.exp_flags & 64) mbar_wait_sleep(&tfull[buf * NH], acc_phase);  // experiment
-        else mbar_wait(&tfull[buf * NH], acc_phase);
+        mbar_wait(&tfull[buf * NH], acc_phase);
         HG_TRACE(it, 1);
         for (int c2 = cluster_id + 1; c2 < c_hi; ++c2) {  // mode 2: wait for the published partials
           int *f = p.sk_flags + c2 * CG + static_cast<int>(rank);
