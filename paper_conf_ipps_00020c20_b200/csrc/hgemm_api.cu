@@ -56,6 +56,9 @@ int env_int(const char *name, int dflt) {
   return e ? std::atoi(e) : dflt;
 }
 const int g_env_stream_rot = env_int("HGEMM_STREAM_ROT", 1);  // streaming kernel k rotation
+const int g_env_stream_stages = env_int("HGEMM_STREAM_STAGES", 0);  // experiments: cap on the streaming ring depth
+const int g_env_stream_g = env_int("HGEMM_STREAM_G", -1);  // streaming kernel k-blocks per stage (3-D Bk map); -1: auto
+const int g_env_stream_mmax = env_int("HGEMM_STREAM_MMAX", 128);  // largest M (= n) the streaming kernel is chosen for
 const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pair kernel (-DHGEMM_ENABLE_MC)
 const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster groups along N
 const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hints
@@ -114,9 +117,10 @@ struct MapKey {
   int64_t ld;
   uint32_t box_inner, box_outer;
   int f32;
+  int g3d;  // 0: the 2-D map; G > 0: the 3-D k-block-grouped view with G k-blocks per box
   bool operator==(const MapKey &o) const {
     return base == o.base && inner == o.inner && outer == o.outer && ld == o.ld && box_inner == o.box_inner &&
-           box_outer == o.box_outer && f32 == o.f32;
+           box_outer == o.box_outer && f32 == o.f32 && g3d == o.g3d;
   }
 };
 constexpr int kMapCache = 32;
@@ -131,7 +135,7 @@ MapCache g_maps;
 
 bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer, int64_t ld, uint32_t box_inner,
               uint32_t box_outer, bool f32 = false) {
-  const MapKey key = {base, inner, outer, ld, box_inner, box_outer, f32 ? 1 : 0};
+  const MapKey key = {base, inner, outer, ld, box_inner, box_outer, f32 ? 1 : 0, 0};
   {
     std::lock_guard<std::mutex> lk(g_maps.mu);
     for (int i = 0; i < kMapCache; ++i)
@@ -156,6 +160,40 @@ bool make_map(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer
   CUresult r = fn(map, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2,
                   const_cast<void *>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                   CU_TENSOR_MAP_SWIZZLE_128B, promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return false;
+  std::lock_guard<std::mutex> lk(g_maps.mu);
+  const int slot = g_maps.next;
+  g_maps.next = (g_maps.next + 1) % kMapCache;
+  g_maps.key[slot] = key;
+  g_maps.map[slot] = *map;
+  g_maps.valid[slot] = true;
+  return true;
+}
+
+// 3-D k-block-grouped view of a K-major FP16 operand (`inner` = K, a multiple
+// of 64; `outer` rows `ld` elements apart): dims {64, outer, K/64}, strides
+// {ld, 128 B}, box {64, box_outer, g}.  One load brings g consecutive k-blocks
+// of box_outer rows as g ordinary SW128 k-block tiles back to back.
+bool make_map_3d(CUtensorMap *map, const void *base, uint64_t inner, uint64_t outer, int64_t ld, uint32_t box_outer,
+                 uint32_t g) {
+  const MapKey key = {base, inner, outer, ld, 64, box_outer, 0, static_cast<int>(g)};
+  {
+    std::lock_guard<std::mutex> lk(g_maps.mu);
+    for (int i = 0; i < kMapCache; ++i)
+      if (g_maps.valid[i] && g_maps.key[i] == key) {
+        *map = g_maps.map[i];
+        return true;
+      }
+  }
+  EncodeTiledFn fn = encode_fn();
+  if (!fn || inner % 64 != 0) return false;
+  cuuint64_t dims[3] = {64, outer, inner / 64};
+  cuuint64_t strides[2] = {static_cast<cuuint64_t>(ld) * 2, 128};
+  cuuint32_t box[3] = {64, box_outer, g};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3, const_cast<void *>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return false;
   std::lock_guard<std::mutex> lk(g_maps.mu);
   const int slot = g_maps.next;
@@ -294,6 +332,20 @@ hgemm_status_t launch_stream(const CUtensorMap &ta, const CUtensorMap &tb, const
   return HGEMM_SUCCESS;
 }
 
+// k-blocks per stage of the streaming kernel (G): G > 1 fetches Bk through the
+// 3-D k-block-grouped map (needs K % 64 == 0 and G | K/64) as long as at least
+// 3 stages of G k-blocks still fit in shared memory (n = 128: G = 2 with 3 stages
+// 32.8 us, G = 1 with 7 stages 34.8 us; profiles/r02/skinny_kgroup_ab.log).
+int stream_kgroup(int64_t k, uint32_t a_bytes, int cw) {
+  if (k % 64 != 0) return 1;
+  const int64_t nkb = k / 64;
+  int g = g_env_stream_g >= 1 ? g_env_stream_g : 2;
+  const uint32_t kb_bytes = a_bytes + static_cast<uint32_t>(cw) * 128u;
+  const uint32_t min_stages = g_env_stream_g >= 1 ? 2u : 3u;
+  while (g > 1 && (nkb % g != 0 || (hg::kStreamSmemBytes - 1536u) / (g * kb_bytes) < min_stages)) g /= 2;
+  return g < 1 ? 1 : g;
+}
+
 // Chunk width for the streaming kernel: the smallest number of chunk waves over
 // the SMs, then the widest chunk (fewest Ak re-reads) among those.
 int stream_chunk(int64_t N, int mt, int num_sms) {
@@ -310,8 +362,12 @@ int stream_chunk(int64_t N, int mt, int num_sms) {
 
 // The streaming kernel takes HBM-bound skinny shapes: M (= n) <= 256 with an
 // N (= m) that gives every SM at least 4 chunk rows of 16.
+// M <= 128 only: at M = 256 the two 16 KB Ak subtiles per k-block leave room for
+// 4 stages (56 KB of HBM loads in flight per SM) and the CTA-pair tile kernel
+// (256-wide tiles, 128 SMs) measured faster: 37.7 vs 44.2 us at 16384 x 256 x 4096
+// (profiles/r02/skinny_kgroup_ab.log).
 inline bool choose_stream(int64_t M, int64_t N, int64_t K, int num_sms) {
-  return M <= 256 && N >= static_cast<int64_t>(num_sms) * 64 && K >= 256;
+  return M <= g_env_stream_mmax && N >= static_cast<int64_t>(num_sms) * 64 && K >= 256;
 }
 
 // Swapped streaming (small m = Ms <= 256, long n = Ns) is available when forced
@@ -551,7 +607,9 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     // covers the 8 KB the M = 128 MMA reads past the 64 real Ak rows
     const uint32_t a_rows = (M <= 64 && cw >= 64) ? 64u : 128u;
     bool ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, a_rows);
-    if (ok) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, cw);
+    const int kg = stream_kgroup(k, a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u, cw);
+    if (ok) ok = kg > 1 ? make_map_3d(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, cw, kg)
+                        : make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, cw);
     if (!ok) return HGEMM_ERR_CUDA;
     hg::StreamParams p = {};
     p.M = static_cast<int32_t>(M);
@@ -561,9 +619,12 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     p.num_chunks = static_cast<int32_t>(cdiv(N, cw));
     p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
     p.a_bytes = a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u;
-    p.stage_bytes = p.a_bytes + static_cast<uint32_t>(cw) * 128u;
+    p.kg = kg;
+    p.b3d = kg > 1 ? 1 : 0;
+    p.stage_bytes = static_cast<uint32_t>(kg) * (p.a_bytes + static_cast<uint32_t>(cw) * 128u);
     p.stages = static_cast<int32_t>(std::min<uint32_t>(hg::kStreamMaxStages,
                                                        (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
+    if (g_env_stream_stages >= 2) p.stages = std::min(p.stages, g_env_stream_stages);
     p.probe = g_probe.load(std::memory_order_relaxed);
     p.k_rot = g_env_stream_rot;
     p.alpha = alpha;
@@ -599,7 +660,9 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     CUtensorMap ta, tb;
     const uint32_t a_rows = (Ms <= 64 && cw >= 64) ? 64u : 128u;
     bool ok = make_map(&ta, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, a_rows);
-    if (ok) ok = make_map(&tb, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, cw);
+    const int kg = stream_kgroup(k, a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u, cw);
+    if (ok) ok = kg > 1 ? make_map_3d(&tb, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, cw, kg)
+                        : make_map(&tb, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, cw);
     if (!ok) return HGEMM_ERR_CUDA;
     hg::StreamParams p = {};
     p.M = static_cast<int32_t>(Ms);
@@ -609,7 +672,9 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     p.num_chunks = static_cast<int32_t>(cdiv(Ns, cw));
     p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
     p.a_bytes = a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u;
-    p.stage_bytes = p.a_bytes + static_cast<uint32_t>(cw) * 128u;
+    p.kg = kg;
+    p.b3d = kg > 1 ? 1 : 0;
+    p.stage_bytes = static_cast<uint32_t>(kg) * (p.a_bytes + static_cast<uint32_t>(cw) * 128u);
     p.stages = static_cast<int32_t>(std::min<uint32_t>(hg::kStreamMaxStages,
                                                        (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
     p.probe = g_probe.load(std::memory_order_relaxed);

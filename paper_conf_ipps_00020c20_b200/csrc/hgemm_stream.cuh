@@ -38,8 +38,9 @@ struct StreamParams {
   int32_t num_chunks;     // ceil(N / cw)
   int32_t num_k_blocks;   // ceil(K / 64)
   int32_t stages;         // ring depth (<= kStreamMaxStages)
-  uint32_t stage_bytes;   // a_bytes + cw * 128, a multiple of 1024
-  uint32_t a_bytes;       // Ak bytes per stage: MT * 16 KB, or 8 KB when M <= 64 (see below)
+  int32_t kg;             // k-blocks per stage (G); > 1 only with the 3-D Bk map (K % 64 == 0, G | nkb)
+  uint32_t stage_bytes;   // G * (a_bytes + cw * 128), a multiple of 1024
+  uint32_t a_bytes;       // Ak bytes per k-block: MT * 16 KB, or 8 KB when M <= 64 (see below)
   int32_t k_rot;          // 1: CTA c walks its k-blocks starting at c * nkb / gridDim (see below)
   float alpha, beta;
   void *D;
@@ -50,6 +51,12 @@ struct StreamParams {
   // resident, computing C = op(A) op(B) with C column-major; each warp's 32 rows
   // are consecutive in memory, so every column store is one 64/128-B segment)
   int32_t tout;
+  // 1: tmB is the 3-D k-block-grouped view of Bk (dims {64, N, K/64}, strides
+  // {ldb, 128 B}, box {64, cw, G}): one TMA load brings G k-blocks of every Bk
+  // row, G x 128 contiguous bytes per row, in the smem image of G ordinary SW128
+  // tiles.  The pure streaming study (tools/stream_study.py --3d) measures
+  // 26.6 us instead of 28.7 us for 128 MiB at G >= 2 (5.04 vs 4.67 TB/s).
+  int32_t b3d;
 };
 
 #ifdef HGEMM_TRACE
@@ -111,22 +118,30 @@ __global__ void __launch_bounds__(192, 1)
   // their op(A) rows (rows are K-contiguous, 2K bytes apart) instead of all
   // hitting the same offset in every row.  Only the summation order changes.
   const int nkb = p.num_k_blocks;
-  const int kb_rot = p.k_rot ? static_cast<int>((static_cast<int64_t>(blockIdx.x) * nkb) / gridDim.x) : 0;
   // TMA producer state (warp 0, lane 0): iteration pi of chunk pch is loaded into stage pstage
   uint32_t pstage = 0, pphase = 0;
   int pch = blockIdx.x, pi = 0;
-  auto produce = [&](int max_loads) {  // issue up to max_loads more k-block loads
+  // Stage layout: [G Ak k-blocks of a_bytes][G Bk k-blocks of cw * 128 B]
+  const int kg = p.kg;
+  const int ngr = nkb / kg;  // k-block groups (stages) per chunk
+  const int gr_rot = p.k_rot ? static_cast<int>((static_cast<int64_t>(blockIdx.x) * ngr) / gridDim.x) : 0;
+  const uint32_t b_off = static_cast<uint32_t>(kg) * a_bytes;
+  const uint32_t b_kb = static_cast<uint32_t>(cw) * 128u;
+  auto produce = [&](int max_loads) {  // issue up to max_loads more stage loads
     for (; pch < p.num_chunks && max_loads > 0; --max_loads) {
-      const int kb = (pi + kb_rot) % nkb;
+      const int kb0 = ((pi + gr_rot) % ngr) * kg;
       mbar_wait(&empty[pstage], pphase ^ 1u);
       const uint32_t sa = smem_u32(smem + pstage * stage_bytes);
       mbar_arrive_expect_tx(&full[pstage], stage_bytes);
       const uint32_t fb = smem_u32(&full[pstage]);
+      for (int j = 0; j < kg; ++j) {
 #pragma unroll
-      for (int t = 0; t < MT; ++t) tma_load_2d(&tmA, sa + t * A_SUB, fb, kb * 64, t * 128, 0);
-      tma_load_2d(&tmB, sa + a_bytes, fb, kb * 64, pch * cw, 0);
+        for (int t = 0; t < MT; ++t) tma_load_2d(&tmA, sa + j * a_bytes + t * A_SUB, fb, (kb0 + j) * 64, t * 128, 0);
+      }
+      if (p.b3d) tma_load_3d(&tmB, sa + b_off, fb, 0, pch * cw, kb0);
+      else tma_load_2d(&tmB, sa + b_off, fb, kb0 * 64, pch * cw, 0);
       if (++pstage == static_cast<uint32_t>(stages)) { pstage = 0; pphase ^= 1u; }
-      if (++pi == nkb) { pi = 0; pch += gridDim.x; }
+      if (++pi == ngr) { pi = 0; pch += gridDim.x; }
     }
   };
   if (warp == 0 && lane == 0) {
@@ -177,19 +192,22 @@ __global__ void __launch_bounds__(192, 1)
         mbar_wait(&tempty[buf], acc_phase ^ 1u);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + buf * 256u;
-        for (int kb = 0; kb < nkb; ++kb) {  // iteration index (the smem stage holds k-block (kb + kb_rot) % nkb)
+        for (int g = 0; g < ngr; ++g) {  // iteration index (the smem stage holds group (g + gr_rot) % ngr)
           mbar_wait(&full[stage], phase);
           tc_fence_after();
-          if (it == 0 && kb == 0) ST_TRACE(2);
-          const uint32_t sa = smem_u32(smem + stage * stage_bytes);
-          const uint32_t sb = sa + a_bytes;
+          if (it == 0 && g == 0) ST_TRACE(2);
+          const uint32_t s0 = smem_u32(smem + stage * stage_bytes);
+          for (int j = 0; j < kg; ++j) {
+            const uint32_t sa = s0 + j * a_bytes;
+            const uint32_t sb = s0 + b_off + j * b_kb;
 #pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            const uint64_t bd = sdesc_k_sw128(sb + k * 32);
+            for (int k = 0; k < 4; ++k) {
+              const uint64_t bd = sdesc_k_sw128(sb + k * 32);
 #pragma unroll
-            for (int t = 0; t < MT; ++t)
-              umma_f16<1>(d_tmem + t * cw, sdesc_k_sw128(sa + t * A_SUB + k * 32), bd, idesc,
-                          (kb | k) != 0 ? 1u : 0u);
+              for (int t = 0; t < MT; ++t)
+                umma_f16<1>(d_tmem + t * cw, sdesc_k_sw128(sa + t * A_SUB + k * 32), bd, idesc,
+                            (g | j | k) != 0 ? 1u : 0u);
+            }
           }
           umma_commit<1>(&empty[stage]);
           if (++stage == static_cast<uint32_t>(stages)) { stage = 0; phase ^= 1u; }

@@ -149,6 +149,16 @@ __device__ __forceinline__ void tma_load_2d(const CUtensorMap *m, uint32_t dst, 
       "l"(reinterpret_cast<uint64_t>(m)), "r"(bar), "r"(c0), "r"(c1), "l"(policy)
       : "memory");
 }
+// 3D tile load (k-block-grouped views: dims {64, rows, k/64}, box {64, rows, G}),
+// completing on a local barrier.
+__device__ __forceinline__ void tma_load_3d(const CUtensorMap *m, uint32_t dst, uint32_t bar, int32_t c0,
+                                            int32_t c1, int32_t c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
+      : "memory");
+}
 // 2D tile load for a CTA pair: data lands in this CTA's shared memory, the
 // transaction bytes complete on `bar_cluster` (the leader CTA's barrier).
 __device__ __forceinline__ void tma_load_2d_pair(const CUtensorMap *m, uint32_t dst, uint32_t bar_cluster,

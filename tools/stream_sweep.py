@@ -17,7 +17,7 @@ w = torch.empty(64 * 1024 * 1024, device="cuda")
 r = torch.zeros(64 * 1024 * 1024, device="cuda")
 
 
-def timed(fn, reps=15):
+def timed(fn, reps=40):
     for _ in range(3):
         fn()
     ts = []
@@ -30,11 +30,17 @@ def timed(fn, reps=15):
         e1.record()
         ts.append((e0, e1))
     torch.cuda.synchronize()
-    return statistics.median(a.elapsed_time(b) for a, b in ts) * 1e3
+    v = [a.elapsed_time(b) * 1e3 for a, b in ts]
+    # the event clock ticks in ~2 us steps on this box: the mean over the reps
+    # resolves differences below one step, the median does not
+    return statistics.mean(v) if "--mean" in sys.argv else statistics.median(v)
 
 
-shapes = [(16384, 64, 4096, 0.0), (16384, 128, 4096, 0.0), (16384, 256, 4096, 0.0),
+shapes = [(16384, 64, 4096, 0.0), (16384, 128, 4096, 0.0), (16384, 256, 4096, 0.0), (16384, 192, 4096, 0.0),
+          (16384, 160, 4096, 0.0), (16384, 96, 4096, 0.0),
           (64, 4096, 2048, 1.0), (256, 4096, 2048, 1.0)]
+if "--skinny" in sys.argv:
+    shapes = shapes[:6]
 for (m, n, k, beta) in shapes:
     A = (torch.rand(m, k, device="cuda") * 2 - 1).half()
     B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
@@ -45,6 +51,14 @@ for (m, n, k, beta) in shapes:
     binding.set_config()
     res = [f"auto {timed(ours):6.1f} ({binding.get_stats()['last_kernel']}/{binding.get_stats()['block_n']})"]
     cws = [16, 32, 48, 64, 96, 112, 128] if min(m, n) <= 256 else []
+    if "--skinny" in sys.argv:
+        cws = [112, 128]
+        if n > 128:
+            for tn in (208, 224, 240, 256):
+                binding.set_config("tc2", block_n=256, tile_n=tn)
+                t = timed(ours)
+                st = binding.get_stats()
+                res.append(f"tc2/256 tile_n {tn} {t:6.1f}" + ("" if st["last_kernel"] == "tc2" else f"[{st['last_kernel']}]"))
     for cw in cws:
         try:
             binding.set_config("stream", block_n=cw)
