@@ -59,6 +59,7 @@ const int g_env_stream_rot = env_int("HGEMM_STREAM_ROT", 1);  // streaming kerne
 const int g_env_stream_stages = env_int("HGEMM_STREAM_STAGES", 0);  // experiments: cap on the streaming ring depth
 const int g_env_stream_g = env_int("HGEMM_STREAM_G", -1);  // streaming kernel k-blocks per stage (3-D Bk map); -1: auto
 const int g_env_stream_mmax = env_int("HGEMM_STREAM_MMAX", 128);  // largest M (= n) the streaming kernel is chosen for
+const int g_env_stream_pre = env_int("HGEMM_STREAM_PRE", 0);    // streaming kernel stage loads before the CTA barrier (0: all)
 const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pair kernel (-DHGEMM_ENABLE_MC)
 const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster groups along N
 const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hints
@@ -316,7 +317,8 @@ hgemm_status_t launch_stream(const CUtensorMap &ta, const CUtensorMap &tb, const
     init.err[dev] = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, hg::kStreamSmemBytes);
   });
   if (init.err[dev] != cudaSuccess) return HGEMM_ERR_CUDA;
-  const uint32_t smem = p.stages * p.stage_bytes + 1024u /*align*/ + 512u /*barriers*/;
+  const uint32_t pad = p.a_bytes == 8192u ? 8192u : 0u;  // hgemm_stream.cuh: 64-row Ak boxes
+  const uint32_t smem = p.stages * p.stage_bytes + pad + 1024u /*align*/ + 512u /*barriers*/;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(static_cast<unsigned>(grid));
   cfg.blockDim = dim3(192);
@@ -342,7 +344,7 @@ int stream_kgroup(int64_t k, uint32_t a_bytes, int cw) {
   int g = g_env_stream_g >= 1 ? g_env_stream_g : 2;
   const uint32_t kb_bytes = a_bytes + static_cast<uint32_t>(cw) * 128u;
   const uint32_t min_stages = g_env_stream_g >= 1 ? 2u : 3u;
-  while (g > 1 && (nkb % g != 0 || (hg::kStreamSmemBytes - 1536u) / (g * kb_bytes) < min_stages)) g /= 2;
+  while (g > 1 && (nkb % g != 0 || (hg::kStreamSmemBytes - 1536u - 8192u) / (g * kb_bytes) < min_stages)) g /= 2;
   return g < 1 ? 1 : g;
 }
 
@@ -376,6 +378,63 @@ inline bool choose_stream(int64_t M, int64_t N, int64_t K, int num_sms) {
 // m = 256: 30.7 vs 16.4 us; profiles/r01b/lstm_swapped_stream.log) -- each
 // 32-row chunk re-reads the resident op(A) k-block by k-block and issues N = 32 MMAs.
 inline bool choose_stream_swapped(int64_t, int64_t, int64_t, int) { return false; }
+
+// One launch of the streaming kernel (hgemm_stream.cuh) on the resident operand
+// R (Ms rows of k, K-contiguous, row pitch ldr; the UMMA A operand, Ak) and the
+// streamed operand S (Ns rows, pitch lds; Bk): D (Ms x Ns) = R S^T, stored at C
+// row-major with pitch ldc, or transposed (tout, the swapped-operand use).
+hgemm_status_t run_stream(const void *R, int64_t ldr, int64_t Ms, const void *S, int64_t lds, int64_t Ns, int64_t k,
+                          float alpha, float beta, void *C, int64_t ldc, bool f32, int tout, const hgemm_config_t &cfg,
+                          int num_sms, int dev, cudaStream_t stream) {
+  const int mt = Ms <= 128 ? 1 : 2;
+  const bool forced_cw = cfg.kernel == HGEMM_KERNEL_STREAM && cfg.block_n;
+  int cw = forced_cw ? cfg.block_n : stream_chunk(Ns, mt, num_sms);
+  if (mt == 2 && cw > 128) cw = 128;
+  // Ak TMA box rows (hgemm_stream.cuh): 64 when Ms <= 64 (the M = 128 MMA reads
+  // 8 KB past the 64 real Ak rows: the next k-block, the stage's Bk or the pad)
+  const uint32_t a_rows = (Ms <= 64) ? 64u : 128u;
+  CUtensorMap ta, tb;
+  bool ok = make_map(&ta, R, static_cast<uint64_t>(k), static_cast<uint64_t>(Ms), ldr, 64, a_rows);
+  const uint32_t a_bytes = a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u;
+  const int kg = stream_kgroup(k, a_bytes, cw);
+  if (ok) ok = kg > 1 ? make_map_3d(&tb, S, static_cast<uint64_t>(k), static_cast<uint64_t>(Ns), lds, cw, kg)
+                      : make_map(&tb, S, static_cast<uint64_t>(k), static_cast<uint64_t>(Ns), lds, 64, cw);
+  if (!ok) return HGEMM_ERR_CUDA;
+  hg::StreamParams p = {};
+  p.M = static_cast<int32_t>(Ms);
+  p.N = static_cast<int32_t>(Ns);
+  p.K = static_cast<int32_t>(k);
+  p.cw = cw;
+  p.num_chunks = static_cast<int32_t>(cdiv(Ns, cw));
+  p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
+  p.a_bytes = a_bytes;
+  p.kg = kg;
+  p.b3d = kg > 1 ? 1 : 0;
+  p.stage_bytes = static_cast<uint32_t>(kg) * (a_bytes + static_cast<uint32_t>(cw) * 128u);
+  p.stages = static_cast<int32_t>(std::min<uint32_t>(
+      hg::kStreamMaxStages, (hg::kStreamSmemBytes - 1536u - (a_rows == 64 ? 8192u : 0u)) / p.stage_bytes));
+  if (g_env_stream_stages >= 2) p.stages = std::min(p.stages, g_env_stream_stages);
+  p.probe = g_probe.load(std::memory_order_relaxed);
+  p.k_rot = tout ? 1 : g_env_stream_rot;
+  p.alpha = alpha;
+  p.beta = beta;
+  p.D = C;
+  p.ldd = ldc;
+  p.tout = tout;
+  p.pre = std::max(1, std::min(p.stages, g_env_stream_pre > 0 ? g_env_stream_pre : p.stages));
+  int grid = static_cast<int>(std::min<int64_t>(p.num_chunks, num_sms));
+  if (cfg.max_ctas > 0) grid = std::min(grid, cfg.max_ctas);
+  hgemm_status_t st;
+  if (mt == 1) st = f32 ? launch_stream<1, true>(ta, tb, p, grid, dev, stream)
+                        : launch_stream<1, false>(ta, tb, p, grid, dev, stream);
+  else st = f32 ? launch_stream<2, true>(ta, tb, p, grid, dev, stream)
+                : launch_stream<2, false>(ta, tb, p, grid, dev, stream);
+  if (st == HGEMM_SUCCESS) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_last = {HGEMM_KERNEL_STREAM, cw, tout /* 1: swapped */, grid, 0, 0};
+  }
+  return st;
+}
 
 inline bool is_t(char c) { return c == 'T' || c == 't'; }
 inline bool is_n(char c) { return c == 'N' || c == 'n'; }
@@ -598,52 +657,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   // ---------------------------------------------------------- HBM streaming (skinny, TN)
   if (!ag && !acc16 && !a_mn && !b_mn && M <= 256 &&
       ((cfg.kernel == HGEMM_KERNEL_STREAM) ||
-       (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream(M, N, k, di.num_sms)))) {
-    const int mt = M <= 128 ? 1 : 2;
-    int cw = cfg.kernel == HGEMM_KERNEL_STREAM && cfg.block_n ? cfg.block_n : stream_chunk(N, mt, di.num_sms);
-    if (mt == 2 && cw > 128) cw = 128;
-    CUtensorMap ta, tb;
-    // Ak TMA box rows (hgemm_stream.cuh): 64 when M <= 64 and the stage's Bk part
-    // covers the 8 KB the M = 128 MMA reads past the 64 real Ak rows
-    const uint32_t a_rows = (M <= 64 && cw >= 64) ? 64u : 128u;
-    bool ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, a_rows);
-    const int kg = stream_kgroup(k, a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u, cw);
-    if (ok) ok = kg > 1 ? make_map_3d(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, cw, kg)
-                        : make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, cw);
-    if (!ok) return HGEMM_ERR_CUDA;
-    hg::StreamParams p = {};
-    p.M = static_cast<int32_t>(M);
-    p.N = static_cast<int32_t>(N);
-    p.K = static_cast<int32_t>(k);
-    p.cw = cw;
-    p.num_chunks = static_cast<int32_t>(cdiv(N, cw));
-    p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
-    p.a_bytes = a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u;
-    p.kg = kg;
-    p.b3d = kg > 1 ? 1 : 0;
-    p.stage_bytes = static_cast<uint32_t>(kg) * (p.a_bytes + static_cast<uint32_t>(cw) * 128u);
-    p.stages = static_cast<int32_t>(std::min<uint32_t>(hg::kStreamMaxStages,
-                                                       (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
-    if (g_env_stream_stages >= 2) p.stages = std::min(p.stages, g_env_stream_stages);
-    p.probe = g_probe.load(std::memory_order_relaxed);
-    p.k_rot = g_env_stream_rot;
-    p.alpha = alpha;
-    p.beta = beta;
-    p.D = C;
-    p.ldd = ldc;
-    int grid = static_cast<int>(std::min<int64_t>(p.num_chunks, di.num_sms));
-    if (cfg.max_ctas > 0) grid = std::min(grid, cfg.max_ctas);
-    hgemm_status_t st;
-    if (mt == 1) st = f32 ? launch_stream<1, true>(ta, tb, p, grid, dev, stream)
-                          : launch_stream<1, false>(ta, tb, p, grid, dev, stream);
-    else st = f32 ? launch_stream<2, true>(ta, tb, p, grid, dev, stream)
-                  : launch_stream<2, false>(ta, tb, p, grid, dev, stream);
-    if (st == HGEMM_SUCCESS) {
-      std::lock_guard<std::mutex> lk(g_mu);
-      g_last = {HGEMM_KERNEL_STREAM, cw, 0, grid, 0, 0};
-    }
-    return st;
-  }
+       (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream(M, N, k, di.num_sms))))
+    return run_stream(B, ldb, M, A, lda, N, k, alpha, beta, C, ldc, f32, 0, cfg, di.num_sms, dev, stream);
 
   // ---------------------------------------------------------- HBM streaming, swapped operands
   // Small m with a long n (LSTM gates, batch <= 256): the big operand is op(B).  The
@@ -652,51 +667,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   // transposed (column-major C, element (i, j) at C + j*ldc + i).
   if (!ag && !acc16 && !a_mn && !b_mn && N <= 256 && M > 256 &&
       ((cfg.kernel == HGEMM_KERNEL_STREAM) ||
-       (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream_swapped(N, M, k, di.num_sms)))) {
-    const int64_t Ms = N, Ns = M;  // the swapped problem: M' = m, N' = n
-    const int mt = Ms <= 128 ? 1 : 2;
-    int cw = cfg.kernel == HGEMM_KERNEL_STREAM && cfg.block_n ? cfg.block_n : stream_chunk(Ns, mt, di.num_sms);
-    if (mt == 2 && cw > 128) cw = 128;
-    CUtensorMap ta, tb;
-    const uint32_t a_rows = (Ms <= 64 && cw >= 64) ? 64u : 128u;
-    bool ok = make_map(&ta, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, a_rows);
-    const int kg = stream_kgroup(k, a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u, cw);
-    if (ok) ok = kg > 1 ? make_map_3d(&tb, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, cw, kg)
-                        : make_map(&tb, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, cw);
-    if (!ok) return HGEMM_ERR_CUDA;
-    hg::StreamParams p = {};
-    p.M = static_cast<int32_t>(Ms);
-    p.N = static_cast<int32_t>(Ns);
-    p.K = static_cast<int32_t>(k);
-    p.cw = cw;
-    p.num_chunks = static_cast<int32_t>(cdiv(Ns, cw));
-    p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
-    p.a_bytes = a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u;
-    p.kg = kg;
-    p.b3d = kg > 1 ? 1 : 0;
-    p.stage_bytes = static_cast<uint32_t>(kg) * (p.a_bytes + static_cast<uint32_t>(cw) * 128u);
-    p.stages = static_cast<int32_t>(std::min<uint32_t>(hg::kStreamMaxStages,
-                                                       (hg::kStreamSmemBytes - 1536u) / p.stage_bytes));
-    p.probe = g_probe.load(std::memory_order_relaxed);
-    p.k_rot = 1;
-    p.alpha = alpha;
-    p.beta = beta;
-    p.D = C;
-    p.ldd = ldc;
-    p.tout = 1;
-    int grid = static_cast<int>(std::min<int64_t>(p.num_chunks, di.num_sms));
-    if (cfg.max_ctas > 0) grid = std::min(grid, cfg.max_ctas);
-    hgemm_status_t st;
-    if (mt == 1) st = f32 ? launch_stream<1, true>(ta, tb, p, grid, dev, stream)
-                          : launch_stream<1, false>(ta, tb, p, grid, dev, stream);
-    else st = f32 ? launch_stream<2, true>(ta, tb, p, grid, dev, stream)
-                  : launch_stream<2, false>(ta, tb, p, grid, dev, stream);
-    if (st == HGEMM_SUCCESS) {
-      std::lock_guard<std::mutex> lk(g_mu);
-      g_last = {HGEMM_KERNEL_STREAM, cw, 1 /* swapped */, grid, 0, 0};
-    }
-    return st;
-  }
+       (cfg.kernel == HGEMM_KERNEL_AUTO && choose_stream_swapped(N, M, k, di.num_sms))))
+    return run_stream(A, lda, N, B, ldb, M, k, alpha, beta, C, ldc, f32, 1, cfg, di.num_sms, dev, stream);
 
   // ---------------------------------------------------------- split-K (under-filled shapes)
   {

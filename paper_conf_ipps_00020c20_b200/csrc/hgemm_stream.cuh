@@ -57,6 +57,7 @@ struct StreamParams {
   // tiles.  The pure streaming study (tools/stream_study.py --3d) measures
   // 26.6 us instead of 28.7 us for 128 MiB at G >= 2 (5.04 vs 4.67 TB/s).
   int32_t b3d;
+  int32_t pre;            // stage loads issued before the CTA barrier (1 .. stages)
 };
 
 #ifdef HGEMM_TRACE
@@ -93,17 +94,21 @@ __global__ void __launch_bounds__(192, 1)
                         const StreamParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
   constexpr uint32_t A_SUB = 128u * 64u * 2u;  // one 128-row Ak subtile of a k-block (16 KB)
-  // M <= 64: the TMA box holds the 64 real Ak rows only (8 KB) and Bk follows
-  // at +8 KB; the M = 128 MMA then reads Bk bytes as Ak rows 64..127, which
+  // M <= 64: the TMA box holds the 64 real Ak rows only (8 KB); the M = 128 MMA
+  // then reads the next 8 KB of shared memory (the next Ak k-block, the stage's
+  // Bk, the next stage or the pad behind the ring) as Ak rows 64..127, which
   // only feed accumulator lanes 64..127 -- rows >= M that are never stored.
-  // One stage shrinks from 30 to 22 KB, so the ring holds 10 instead of 7.
+  // One k-block shrinks from 30 to 22 KB (n = 64, cw = 112), 20 to 12 KB (m = 64, cw = 32).
   const uint32_t a_bytes = p.a_bytes;
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw_u32 = smem_u32(smem_raw);
   uint8_t *smem = smem_raw + ((1024u - (raw_u32 & 1023u)) & 1023u);
   const int stages = p.stages;
   const uint32_t stage_bytes = p.stage_bytes;
-  uint64_t *full = reinterpret_cast<uint64_t *>(smem + stages * stage_bytes);
+  // M <= 64 (8 KB Ak boxes): the last Ak tile's MMA reads 8 KB past its box, so the
+  // barriers sit behind an 8 KB pad after the ring (the host sizes the allocation)
+  const uint32_t pad = a_bytes == 8192u ? 8192u : 0u;
+  uint64_t *full = reinterpret_cast<uint64_t *>(smem + stages * stage_bytes + pad);
   uint64_t *empty = full + kStreamMaxStages;
   uint64_t *tfull = empty + kStreamMaxStages;  // [2]
   uint64_t *tempty = tfull + 2;                // [2]
@@ -156,7 +161,11 @@ __global__ void __launch_bounds__(192, 1)
     }
     fence_mbarrier_init();
     griddep_wait();
-    produce(stages);
+    // p.pre (<= stages) stage loads before the CTA barrier: TMA issue stalls once the
+    // engine's queue is full, and the MMA warp waits at the barrier behind it
+    // (tools/trace_stream.py: with 16 stages issued here the first MMA started 5 us
+    // after the kernel, 0.3 us after its data)
+    produce(p.pre);
   }
   if (warp == 1) {
     if (lane == 0) {

@@ -52,7 +52,7 @@ for (m, n, k, beta) in shapes:
     res = [f"auto {timed(ours):6.1f} ({binding.get_stats()['last_kernel']}/{binding.get_stats()['block_n']})"]
     cws = [16, 32, 48, 64, 96, 112, 128] if min(m, n) <= 256 else []
     if "--skinny" in sys.argv:
-        cws = [112, 128]
+        cws = [112]
         if n > 128:
             for tn in (208, 224, 240, 256):
                 binding.set_config("tc2", block_n=256, tile_n=tn)
