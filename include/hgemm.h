@@ -154,7 +154,12 @@ typedef enum {
                                     each owning column chunks of C^T of block_n (multiple of 16) rows of op(A);
                                     with n > 256 and m <= 256 the operands are swapped (op(B) streamed,
                                     C stored transposed; reported with group_m = 1);
-                                    other shapes/layouts fall back to the automatic choice */
+                                    other shapes/layouts fall back to the automatic choice.  The
+                                    automatic choice takes it for n <= 128 and m >= 64 x #SMs
+                                    (16384 x 256 runs faster on the 2-SM tile kernel).  With K a
+                                    multiple of 64 a stage holds G consecutive k-blocks of op(A)
+                                    fetched by one 3-D TMA load; hgemm_get_last_config reports G in
+                                    `splits` */
 } hgemm_kernel_t;
 
 typedef struct {
@@ -180,8 +185,10 @@ typedef struct {
                           16 in [128, 256] (0 = block_n).  Tiles of tile_n columns of the output's
                           contiguous dimension (m), so that the tile count fills whole waves; needs a
                           K-major op(A) (transA 'T'), otherwise block_n is used.  The automatic choice
-                          picks it by the wave model; hgemm_get_last_config reports the width used
-                          (0 = block_n).  Whole tiles, no stream-K. */
+                          does not use it (measured slower than 256-wide tiles with stream-K at every
+                          mid-size shape tried; environment HGEMM_FLEX=1 lets its wave model consider
+                          it); hgemm_get_last_config reports the width used (0 = block_n).  Whole
+                          tiles, no stream-K. */
 } hgemm_config_t;
 
 /* Set (cfg != NULL) or reset to automatic (cfg == NULL) the process-global

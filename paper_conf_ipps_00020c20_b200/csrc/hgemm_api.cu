@@ -431,7 +431,7 @@ hgemm_status_t run_stream(const void *R, int64_t ldr, int64_t Ms, const void *S,
                 : launch_stream<2, false>(ta, tb, p, grid, dev, stream);
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);
-    g_last = {HGEMM_KERNEL_STREAM, cw, tout /* 1: swapped */, grid, 0, 0};
+    g_last = {HGEMM_KERNEL_STREAM, cw, tout /* 1: swapped */, grid, kg /* k-blocks per stage */, 0};
   }
   return st;
 }

@@ -455,6 +455,45 @@ def test_stream_kernel_integer_exact(oracle_mod, n):
     assert case.stats["last_kernel"] == "stream", case.stats
 
 
+@pytest.mark.parametrize("n", [64, 100, 128])
+@pytest.mark.parametrize("k,g", [(640, 2), (704, 1), (4096, 2)])
+@pytest.mark.parametrize("cw,max_ctas", [(112, 0), (48, 5)])
+@pytest.mark.parametrize("out,beta", [("f16", 0.5), ("f32", 0.0)])
+def test_stream_kernel_kgroup(oracle_mod, n, k, g, cw, max_ctas, out, beta):
+    """Streaming kernel with K a multiple of 64: G = 2 consecutive k-blocks per stage
+    through the 3-D op(A) tensor map when G divides the k-block count (640, 4096),
+    G = 1 through the 2-D map when it does not (704 = 11 k-blocks); ragged m, several
+    chunks per CTA (max_ctas), k rotation across CTAs."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("stream", block_n=cw, max_ctas=max_ctas)
+    m = 1003
+    C = inputs.uniform_f16(m, n, 57).astype(np.float32 if out == "f32" else np.float16)
+    case = GpuCase(inputs.uniform_f16(m, k, 55), inputs.uniform_f16(k, n, 56), "T", "N", 0.75, beta, C=C,
+                   out=out, pad=(8, 16, 8))
+    got = case.run_gpu()
+    assert case.stats["last_kernel"] == "stream", case.stats
+    assert case.stats["splits"] == g, case.stats
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, got, r, ab)
+    assert np.all(np.isnan(case.padding(got).astype(np.float32)))
+
+
+def test_stream_routing_by_n(oracle_mod):
+    """Automatic choice on the skinny TN shapes: n <= 128 streams, n in (128, 256] takes
+    the 2-SM tile kernel (faster there); both against the oracle on sampled entries."""
+    m, k = 16384, 512
+    for n, expect in ((96, "stream"), (128, "stream"), (192, "tc2"), (256, "tc2")):
+        case = GpuCase(inputs.uniform_f16(m, k, 61), inputs.uniform_f16(k, n, 62), "T", "N", out="f16")
+        got = case.run_gpu()
+        assert case.stats["last_kernel"] == expect, (n, case.stats)
+        rows = np.arange(0, m, 89)
+        ii, jj = np.meshgrid(rows, np.arange(n), indexing="ij")
+        _, r, ab = oracle_mod.hgemm_ref_entries(m, n, k, 1.0, case.A, case.lda, case.B, case.ldb, 0.0, None,
+                                                case.ldc, "T", "N", "f16", ii.ravel(), jj.ravel())
+        g = case.view(got)[ii.ravel(), jj.ravel()].astype(np.float64)
+        assert np.all(np.abs(g - r) <= 1e-3 * ab + ulp16(np.maximum(np.abs(g), np.abs(r))))
+
+
 def test_stream_kernel_auto_and_fallback(oracle_mod):
     """Automatic choice: the skinny TN shape of BJ configs[3] takes the streaming
     kernel; the same shape in NN layout takes the tile kernels (still correct)."""
