@@ -59,6 +59,7 @@ const int g_env_stream_rot = env_int("HGEMM_STREAM_ROT", 1);  // streaming kerne
 const int g_env_stream_stages = env_int("HGEMM_STREAM_STAGES", 0);  // experiments: cap on the streaming ring depth
 const int g_env_stream_g = env_int("HGEMM_STREAM_G", -1);  // streaming kernel k-blocks per stage (3-D Bk map); -1: auto
 const int g_env_stream_mmax = env_int("HGEMM_STREAM_MMAX", 128);  // largest M (= n) the streaming kernel is chosen for
+const int g_env_sk_kg = env_int("HGEMM_SK_KG", 2);            // split-K kernel k-blocks per stage (1 or 2)
 const int g_env_stream_pre = env_int("HGEMM_STREAM_PRE", 0);    // streaming kernel stage loads before the CTA barrier (0: all)
 const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pair kernel (-DHGEMM_ENABLE_MC)
 const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster groups along N
@@ -686,7 +687,12 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     if (use_sk) {
       CUtensorMap ta, tb;
       bool ok;
-      if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
+      // k-groups of 2 (3-D Ak view, one load of 256 contiguous bytes per Ak row): K-major Ak,
+      // K % 64 == 0 and every split's k range a whole number of groups
+      const int nkb_all = static_cast<int>(cdiv(k, 64));
+      const int sk_kg = (!a_mn && k % 64 == 0 && nkb_all % (2 * sk_spl) == 0 && g_env_sk_kg == 2) ? 2 : 1;
+      if (!a_mn) ok = sk_kg == 2 ? make_map_3d(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 128, 2)
+                                 : make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
       else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
       if (ok) {
         if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, sk_bn);
@@ -701,6 +707,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
       p.num_n_tiles = static_cast<int32_t>(cdiv(N, sk_bn));
       p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
       p.group_m = p.num_m_tiles;  // tiles in m-fastest order
+      p.sk_kg = sk_kg;
       p.alpha = alpha;
       p.beta = beta;
       p.D = C;

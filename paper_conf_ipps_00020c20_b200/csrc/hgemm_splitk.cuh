@@ -132,29 +132,41 @@ __global__ void __launch_bounds__(192, 1)
   // TMA producer state (warp 0, lane 0): k-block pkb is loaded into ring stage pstage
   const int a_row = tm * BM;
   const int b_row = tn * BN;
+  // k-groups (p.sk_kg = G = 1 or 2, the host guarantees G | nkb): a ring stage holds G
+  // consecutive k-blocks, [G Ak k-blocks][G Bk k-blocks]; with G = 2 the Ak k-blocks come
+  // from ONE 3-D TMA load (tmA = the k-group view, box {64, 128, 2}), 256 contiguous bytes
+  // per Ak row (HBM streaming).  The ring keeps its size:
+  // STAGES / G stages of G * STAGE_BYTES.
+  const int kg = (!A_MN && p.sk_kg == 2) ? 2 : 1;
+  const int nst = STAGES / kg;
+  const uint32_t sst_bytes = static_cast<uint32_t>(kg) * STAGE_BYTES;
   uint32_t pstage = 0, pphase = 0;
   int pkb = kb0;
-  auto produce = [&](int upto) {  // issue the loads of k-blocks [pkb, upto)
-    for (; pkb < upto; ++pkb) {
+  auto produce = [&](int upto) {  // issue the loads of k-blocks [pkb, upto), G per stage
+    for (; pkb < upto; pkb += kg) {
       mbar_wait(&empty[pstage], pphase ^ 1u);
-      const uint32_t sa = smem_u32(smem + pstage * STAGE_BYTES);
-      const uint32_t sb = sa + A_BYTES;
-      mbar_arrive_expect_tx(&full[pstage], STAGE_BYTES);
+      const uint32_t sa = smem_u32(smem + pstage * sst_bytes);
+      const uint32_t sb = sa + kg * A_BYTES;
+      mbar_arrive_expect_tx(&full[pstage], sst_bytes);
       const uint32_t fb = smem_u32(&full[pstage]);
       const int k0 = pkb * BK;
       if constexpr (!A_MN) {
-        tma_load_2d(&tmA, sa, fb, k0, a_row, 0);
+        if (kg == 2) tma_load_3d(&tmA, sa, fb, 0, a_row, pkb);
+        else tma_load_2d(&tmA, sa, fb, k0, a_row, 0);
       } else {
 #pragma unroll
         for (int q = 0; q < BM / 64; ++q) tma_load_2d(&tmA, sa + q * 8192, fb, a_row + 64 * q, k0, 0);
       }
-      if constexpr (!B_MN) {
-        tma_load_2d(&tmB, sb, fb, k0, b_row, 0);
-      } else {
+      for (int j = 0; j < kg; ++j) {
+        if constexpr (!B_MN) {
+          tma_load_2d(&tmB, sb + j * SH::B_BYTES, fb, k0 + j * BK, b_row, 0);
+        } else {
 #pragma unroll
-        for (int q = 0; q < BN / 64; ++q) tma_load_2d(&tmB, sb + q * 8192, fb, b_row + 64 * q, k0, 0);
+          for (int q = 0; q < BN / 64; ++q)
+            tma_load_2d(&tmB, sb + j * SH::B_BYTES + q * 8192, fb, b_row + 64 * q, k0 + j * BK, 0);
+        }
       }
-      if (++pstage == STAGES) { pstage = 0; pphase ^= 1u; }
+      if (++pstage == static_cast<uint32_t>(nst)) { pstage = 0; pphase ^= 1u; }
     }
   };
   if (warp == 0 && lane == 0) {
@@ -163,13 +175,13 @@ __global__ void __launch_bounds__(192, 1)
     // overlaps the TMEM allocation and the CTA barrier below.
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
-    for (int s = 0; s < STAGES; ++s) {
+    for (int s = 0; s < nst; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
     fence_mbarrier_init();
     griddep_wait();
-    produce(min(kb1, kb0 + STAGES));
+    produce(min(kb1, kb0 + nst * kg));
   }
   if (warp == 1) {
     if (lane == 0) {
@@ -225,22 +237,25 @@ __global__ void __launch_bounds__(192, 1)
     // ------------------------------------------------------------ MMA issuer
     if (lane == 0) {
       uint32_t stage = 0, phase = 0;
-      for (int j = 0; j < nkb; ++j) {
+      for (int j = 0; j < nkb; j += kg) {
         mbar_wait(&full[stage], phase);
         tc_fence_after();
         if (j == 0) SK_TRACE(2);
-        const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
-        const uint32_t sb = sa + A_BYTES;
+        const uint32_t s0 = smem_u32(smem + stage * sst_bytes);
+        for (int jj = 0; jj < kg; ++jj) {
+          const uint32_t sa = s0 + jj * A_BYTES;
+          const uint32_t sb = s0 + kg * A_BYTES + jj * SH::B_BYTES;
 #pragma unroll
-        for (int k = 0; k < BK / 16; ++k) {
-          const uint32_t a_addr = sa + k * A_KSTEP;
-          const uint32_t b_addr = sb + k * B_KSTEP;
-          const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
-          const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
-          umma_f16<1>(tmem_base, ad, bd, IDESC, (j | k) != 0 ? 1u : 0u);
+          for (int k = 0; k < BK / 16; ++k) {
+            const uint32_t a_addr = sa + k * A_KSTEP;
+            const uint32_t b_addr = sb + k * B_KSTEP;
+            const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
+            const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
+            umma_f16<1>(tmem_base, ad, bd, IDESC, (j | jj | k) != 0 ? 1u : 0u);
+          }
         }
         umma_commit<1>(&empty[stage]);
-        if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+        if (++stage == static_cast<uint32_t>(nst)) { stage = 0; phase ^= 1u; }
       }
       SK_TRACE(3);
       if (nkb > 0) umma_commit<1>(tfull);

@@ -97,6 +97,7 @@ struct TcParams {
   int32_t exp_flags;  // experiments (HGEMM_EXP): 1 = no ring staging for the last item, 2 = no C-load hold-back,
                       // 4 = wait for store completion before exit, 8 = no PDL trigger, 16 = no cluster
                       // attribute for 1-CTA launches (host side)
+  int32_t sk_kg;      // split-K kernel: k-blocks per ring stage (1, or 2 with tmA the 3-D k-group view)
 };
 
 // One unit of work of a cluster: k-blocks [kb0, kb1) of cluster tile `tile`.

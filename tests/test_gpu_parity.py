@@ -314,10 +314,11 @@ def test_stream_k_graph_capture(oracle_mod):
 @pytest.mark.parametrize("bn", [64, 128])
 @pytest.mark.parametrize("tA,tB", TRANS)
 def test_splitk_splits(oracle_mod, splits, bn, tA, tB):
-    """Split-K over a cluster: every split count, ragged K ranges (some splits empty)."""
+    """Split-K over a cluster: every split count, ragged K ranges (some splits empty);
+    k = 1024 (16 k-blocks) takes the 2-k-block stages (3-D Ak view) for a K-major op(B)^T."""
     from paper_conf_ipps_00020c20_b200 import binding
     binding.set_config("splitk", block_n=bn, splits=splits)
-    for (m, n, k) in [(200, 300, 1000), (64, 4096, 448), (130, 257, 100)]:
+    for (m, n, k) in [(200, 300, 1000), (64, 4096, 448), (130, 257, 100), (72, 1000, 1024)]:
         case = GpuCase(inputs.uniform_f16(m, k, 7), inputs.uniform_f16(k, n, 8), tA, tB, 1.0, 0.5,
                        C=inputs.uniform_f16(m, n, 9), out="f16")
         got = case.run_gpu()
@@ -326,12 +327,13 @@ def test_splitk_splits(oracle_mod, splits, bn, tA, tB):
         assert_within_tolerance(case, got, r, ab)
         a, b = case.run_gpu(repeat=2)
         assert np.array_equal(a.view(np.uint16), b.view(np.uint16))   # deterministic reduction order
-    opA = inputs.integer_f16(90, 640, 3, -4, 4)
-    opB = inputs.integer_f16(640, 70, 4, -4, 4)
-    case = GpuCase(opA, opB, tA, tB, out="f32")
-    got = case.view(case.run_gpu())
-    _, r, _ = case.oracle(oracle_mod)
-    assert np.array_equal(got.astype(np.float64), r)
+    for kk in (640, 2048):
+        opA = inputs.integer_f16(90, kk, 3, -4, 4)
+        opB = inputs.integer_f16(kk, 70, 4, -4, 4)
+        case = GpuCase(opA, opB, tA, tB, out="f32")
+        got = case.view(case.run_gpu())
+        _, r, _ = case.oracle(oracle_mod)
+        assert np.array_equal(got.astype(np.float64), r)
 
 
 def test_splitk_auto_for_underfilled(oracle_mod):

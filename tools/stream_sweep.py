@@ -41,6 +41,8 @@ shapes = [(16384, 64, 4096, 0.0), (16384, 128, 4096, 0.0), (16384, 256, 4096, 0.
           (64, 4096, 2048, 1.0), (256, 4096, 2048, 1.0)]
 if "--skinny" in sys.argv:
     shapes = shapes[:6]
+if "--lstm" in sys.argv:
+    shapes = shapes[6:]
 for (m, n, k, beta) in shapes:
     A = (torch.rand(m, k, device="cuda") * 2 - 1).half()
     B = (torch.rand(n, k, device="cuda") * 2 - 1).half()
@@ -50,7 +52,7 @@ for (m, n, k, beta) in shapes:
         binding.hgemm(m, n, k, 1.0, A, k, B, k, beta, C, m, "T", "N", "f16")
     binding.set_config()
     res = [f"auto {timed(ours):6.1f} ({binding.get_stats()['last_kernel']}/{binding.get_stats()['block_n']})"]
-    cws = [16, 32, 48, 64, 96, 112, 128] if min(m, n) <= 256 else []
+    cws = [16, 32, 48, 64, 96, 112, 128] if min(m, n) <= 256 and "--lstm" not in sys.argv else []
     if "--skinny" in sys.argv:
         cws = [112]
         if n > 128:
