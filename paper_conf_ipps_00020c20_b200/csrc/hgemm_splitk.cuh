@@ -36,7 +36,9 @@ struct SkShape {
   static constexpr uint32_t A_BYTES = BM * BK * 2;
   static constexpr uint32_t B_BYTES = BN * BK * 2;
   static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr uint32_t PART_BYTES = BM * BN * 4;     // receive buffer: S x 128 rows x BN/S FP32
+  // receive buffer: (S-1) peer slots x 128 rows x BN/S FP32 (peer src lands in slot
+  // src < rank ? src : src - 1; the owner's own slice stays in registers)
+  static constexpr uint32_t PART_BYTES = (S - 1) * BM * (BN / S) * 4;
   static constexpr int STAGES_FIT = static_cast<int>((227u * 1024u - PART_BYTES - 2048u) / STAGE_BYTES);
   // At most 6 stages: 8 for BN = 64 (every k-block of an LSTM-gate CTA in flight at once) fit
   // but measured 0.9 us slower per launch (profiles/r02/splitk_stages_sweep.log)
@@ -48,10 +50,11 @@ struct SkShape {
   static_assert(S == 2 || S == 4 || S == 8, "S");
   static_assert(SLICE % 8 == 0, "slice");
   static_assert(STAGES >= 2, "stages");
-  static_assert(PART_BYTES <= STAGES * STAGE_BYTES, "reduction staging in the smem ring");
+  static_assert(BM * BN * 4 <= STAGES * STAGE_BYTES, "reduction staging ([owner][row][SLICE]) in the smem ring");
 };
 
-// Receive buffer of the owner CTA: [S sources][128 rows][SLICE FP32], the
+// Receive buffer of the owner CTA: [S-1 peer slots][128 rows][SLICE FP32] (the
+// sender stages in the same layout with S owner slots), the
 // 16-byte chunk index of a row rotated by the row so that consecutive rows
 // (threads) writing or reading the same chunk use different bank groups.
 template <int SLICE>
@@ -310,7 +313,8 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll 1
       for (uint32_t o = 0; o < static_cast<uint32_t>(S); ++o) {
         if (o == rank) continue;
-        bulk_copy_s2cluster(mapa_shared(smem_u32(part) + rank * SLAB + rows_off, o), stg + o * SLAB + rows_off,
+        const uint32_t slot = rank < o ? rank : rank - 1u;  // this CTA's slot in owner o's buffer
+        bulk_copy_s2cluster(mapa_shared(smem_u32(part) + slot * SLAB + rows_off, o), stg + o * SLAB + rows_off,
                             32u * SLICE * 4u, mapa_shared(smem_u32(rbar), o));
       }
     }
@@ -333,7 +337,8 @@ __global__ void __launch_bounds__(192, 1)
       }
 #pragma unroll
       for (int q = 0; q < SLICE / 4; ++q) {
-        const float4 v = ld_shared_f4(rbuf + recv_off(static_cast<uint32_t>(src), prow, q));
+        const uint32_t slot = static_cast<uint32_t>(src) < rank ? static_cast<uint32_t>(src) : static_cast<uint32_t>(src) - 1u;
+        const float4 v = ld_shared_f4(rbuf + recv_off(slot, prow, q));
         acc[4 * q + 0] += v.x;
         acc[4 * q + 1] += v.y;
         acc[4 * q + 2] += v.z;
