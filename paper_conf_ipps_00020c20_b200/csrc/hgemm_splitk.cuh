@@ -126,9 +126,24 @@ __global__ void __launch_bounds__(192, 1)
   do {                                                                                         \
     if (p.probe != nullptr && blockIdx.x < 256) p.probe[8 + 8 * blockIdx.x + (f)] = globaltimer_ns(); \
   } while (0)
+// prologue detail (second region): p.probe[8 + 2048 + 8*blockIdx.x + f]
+#define SK_TRACE2(f)                                                                           \
+  do {                                                                                         \
+    if (p.probe != nullptr && blockIdx.x < 256) p.probe[8 + 2048 + 8 * blockIdx.x + (f)] = globaltimer_ns(); \
+  } while (0)
+#define SK_TRACE3(f)                                                                           \
+  do {                                                                                         \
+    if (p.probe != nullptr && blockIdx.x < 256) p.probe[8 + 4096 + 8 * blockIdx.x + (f)] = globaltimer_ns(); \
+  } while (0)
 #else
+#define SK_TRACE3(f) \
+  do {               \
+  } while (0)
 #define SK_TRACE(f) \
   do {              \
+  } while (0)
+#define SK_TRACE2(f) \
+  do {               \
   } while (0)
 #endif
   if (threadIdx.x == 0) SK_TRACE(0);
@@ -169,6 +184,9 @@ __global__ void __launch_bounds__(192, 1)
             tma_load_2d(&tmB, sb + j * SH::B_BYTES + q * 8192, fb, b_row + 64 * q, k0 + j * BK, 0);
         }
       }
+#ifdef HGEMM_TRACE
+      if (pkb == kb0) SK_TRACE2(6);
+#endif
       if (++pstage == static_cast<uint32_t>(nst)) { pstage = 0; pphase ^= 1u; }
     }
   };
@@ -176,6 +194,7 @@ __global__ void __launch_bounds__(192, 1)
     // The producer initialises the ring barriers itself and issues the first ring of
     // loads right away (after griddepcontrol.wait), so the first HBM round trip
     // overlaps the TMEM allocation and the CTA barrier below.
+    SK_TRACE2(0);
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
     for (int s = 0; s < nst; ++s) {
@@ -183,8 +202,11 @@ __global__ void __launch_bounds__(192, 1)
       mbar_init(&empty[s], 1);
     }
     fence_mbarrier_init();
+    SK_TRACE2(1);
     griddep_wait();
+    SK_TRACE2(2);
     produce(min(kb1, kb0 + nst * kg));
+    SK_TRACE2(3);
   }
   if (warp == 1) {
     if (lane == 0) {
@@ -196,11 +218,16 @@ __global__ void __launch_bounds__(192, 1)
       fence_mbarrier_init();
     }
     __syncwarp();
+    if (lane == 0) SK_TRACE2(4);
     tmem_alloc<1>(smem_u32(tmem_slot), SH::TMEM_COLS);
+    if (lane == 0) SK_TRACE2(5);
   }
   __syncwarp();
+  if (lane == 0 && warp == 2) SK_TRACE3(0);
+  if (lane == 0 && warp == 5) SK_TRACE3(1);
   tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0) SK_TRACE3(2);
   tc_fence_after();
   // Cluster barrier, split: every thread arrives now (its barriers are initialised); a
   // thread waits only before its first access to a peer's shared memory (the epilogue's
@@ -232,6 +259,7 @@ __global__ void __launch_bounds__(192, 1)
       }
     }
   }
+  if (lane == 0 && warp == 2) SK_TRACE3(3);
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer (the rest of the k range)

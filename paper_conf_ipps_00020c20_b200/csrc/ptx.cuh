@@ -407,13 +407,23 @@ __device__ __forceinline__ void griddep_launch_dependents() {
 }
 
 // ------------------------------------------------------------------ cluster
+// The arrivals are relaxed: no cluster barrier of the kernels publishes generic memory
+// writes (mbarrier initialisation is published by fence.mbarrier_init.release.cluster,
+// shared-memory data by the mbarrier transactions and explicit fences; the waits keep
+// acquire).  A release arrival waits until the thread's earlier memory operations are
+// performed: in the split-K prologue that held every CTA ~3 us on a cold L2 before its
+// first MMA (profiles/r02/trace_splitk_prologue.log).  -DHGEMM_CLUSTER_RELEASE restores it
+// (experiments).
+#ifdef HGEMM_CLUSTER_RELEASE
+#define HG_CLUSTER_ARRIVE "barrier.cluster.arrive.release.aligned;"
+#else
+#define HG_CLUSTER_ARRIVE "barrier.cluster.arrive.relaxed.aligned;"
+#endif
 __device__ __forceinline__ void cluster_sync() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+  asm volatile(HG_CLUSTER_ARRIVE "\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 // Split phases of the cluster barrier (every thread of the cluster arrives once per phase).
-__device__ __forceinline__ void cluster_arrive() {
-  asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
-}
+__device__ __forceinline__ void cluster_arrive() { asm volatile(HG_CLUSTER_ARRIVE ::: "memory"); }
 __device__ __forceinline__ void cluster_wait() { asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory"); }
 // Bulk copy of `bytes` (multiple of 16) from this CTA's shared memory to a peer CTA's
 // shared memory (shared::cluster addresses of the destination and of its mbarrier),
