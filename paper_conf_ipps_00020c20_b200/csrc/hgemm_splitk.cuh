@@ -64,6 +64,15 @@ __device__ __forceinline__ uint32_t recv_off_t(uint32_t src, uint32_t row, uint3
   return (src * 128u + row) * (SLICE * 4u) + q * 16u;
 }
 
+// 16 bytes from registers into a peer CTA's shared memory, completing 16 bytes of
+// transaction count on the peer's mbarrier (both shared::cluster addresses).
+__device__ __forceinline__ void st_async_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t c, uint32_t d,
+                                            uint32_t mbar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];"
+               ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d), "r"(mbar)
+               : "memory");
+}
+
 __device__ __forceinline__ void st_shared_cluster_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t c,
                                                      uint32_t d) {
   asm volatile("st.shared::cluster.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d)
@@ -305,6 +314,12 @@ __global__ void __launch_bounds__(192, 1)
     const uint32_t prow = quad * 32u + lane;  // TMEM lane == tile row
     const uint32_t stg = smem_u32(smem);      // staging: [owner][row][SLICE] (recv_off layout)
     float own[SLICE];
+    // exp_flags & 64 (experiment): push each 16-B chunk of a peer's slice straight from
+    // registers into the owner's receive buffer (st.async, completing on its rbar) instead
+    // of staging the slices locally and sending them with bulk copies
+    const bool direct = (p.exp_flags & 64) != 0;
+    if (direct) cluster_wait();  // every peer's rbar is initialised before we store into it
+    const uint32_t part_u32 = smem_u32(part), rbar_u32 = smem_u32(rbar);
     mbar_wait(tfull, 0);
     tc_fence_after();
     if (warp == 2 && lane == 0) SK_TRACE(4);
@@ -314,6 +329,7 @@ __global__ void __launch_bounds__(192, 1)
       if (nkb > 0) {
         tmem_ld_32x32b_x32(tmem_base + ((quad * 32u) << 16) + c * 32, v);
         tmem_ld_wait();
+        if (c == 0 && warp == 2 && lane == 0) SK_TRACE3(4);
       } else {
 #pragma unroll
         for (int j = 0; j < 32; ++j) v[j] = 0u;
@@ -326,17 +342,24 @@ __global__ void __launch_bounds__(192, 1)
         if (owner == rank) {
 #pragma unroll
           for (int e = 0; e < 4; ++e) own[(colq % SLICE) + e] = __uint_as_float(v[4 * q + e]);
+        } else if (direct) {
+          const uint32_t slot = rank < owner ? rank : rank - 1u;
+          st_async_v4(mapa_shared(part_u32 + recv_off(slot, prow, within), owner), v[4 * q], v[4 * q + 1],
+                      v[4 * q + 2], v[4 * q + 3], mapa_shared(rbar_u32, owner));
         } else {
           st_shared_v4(stg + owner * SLAB + recv_off(0u, prow, within), v[4 * q], v[4 * q + 1], v[4 * q + 2],
                        v[4 * q + 3]);
         }
       }
     }
+    if (warp == 2 && lane == 0) SK_TRACE3(5);
     tc_fence_before();
+    if (!direct) {
     fence_proxy_async_smem();  // the staged slices -> the bulk copies (async proxy)
     __syncwarp();
     cluster_wait();            // every peer's rbar is initialised before we copy into it
-    if (lane == 0) {
+    }
+    if (lane == 0 && !direct) {
       const uint32_t rows_off = quad * 32u * SLICE * 4u;  // this warp's 32 rows in a slice block
 #pragma unroll 1
       for (uint32_t o = 0; o < static_cast<uint32_t>(S); ++o) {
@@ -353,6 +376,7 @@ __global__ void __launch_bounds__(192, 1)
     const int col0 = tn * BN + static_cast<int>(rank) * SLICE;
     const uint32_t rbuf = smem_u32(part);
     if constexpr (S > 1) mbar_wait(rbar, 0);  // the (S-1) peers' slices have landed
+    if (warp == 2 && lane == 0) SK_TRACE3(6);
     float acc[SLICE];
 #pragma unroll
     for (int j = 0; j < SLICE; ++j) acc[j] = 0.0f;
@@ -373,6 +397,7 @@ __global__ void __launch_bounds__(192, 1)
         acc[4 * q + 3] += v.w;
       }
     }
+    if (warp == 2 && lane == 0) SK_TRACE3(7);
     if (row < p.M) {
       const float alpha = p.alpha, beta = p.beta;
       if constexpr (OUT_F32) {

@@ -523,10 +523,23 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
   const uint16_t pair_mask = static_cast<uint16_t>(((1u << CG) - 1u) << leader);
   const uint16_t empty_mask = static_cast<uint16_t>(MC == 2 ? 0xFu : pair_mask);
   
+  // The producer's first work item and its PDL wait are settled here, overlapping warp 1's
+  // barrier initialisation and TMEM allocation, so that the first operand loads issue right
+  // after the CTA (pair) barrier (cold 256^3: the item arithmetic and its parameter reads
+  // took ~0.45 us between the barrier and the first TMA; profiles/r02/trace_tc_prologue.log).
+  WorkItem wi0{0, 0, 0};
+  bool has0 = false;
+  int tile0 = 0, sub0 = -1, tm0 = 0, tn0 = 0;
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
     tma_prefetch_desc(&tmD);
+    has0 = get_item(p, cluster_id, num_clusters, 0, wi0);
+    if (has0) {
+      item_tile(p, wi0.tile, tile0, sub0);
+      tile_coords(tile0, p, tm0, tn0);
+    }
+    griddep_wait();  // the producer's first global access follows the barrier below
   }
   if (warp == 1) {
     if (lane == 0) {
@@ -581,10 +594,12 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
         const int target = ++nbar * static_cast<int>(gridDim.x);
         while (ld_acquire_gpu(p.wsync) < target) __nanosleep(64);
       };
-      for (int i = 0; get_item(p, cluster_id, num_clusters, i, wi); ++i) {
-        int tm, tn, tile, sub;
-        item_tile(p, wi.tile, tile, sub);
-        tile_coords(tile, p, tm, tn);
+      for (int i = 0; i == 0 ? (wi = wi0, has0) : get_item(p, cluster_id, num_clusters, i, wi); ++i) {
+        int tm = tm0, tn = tn0, tile = tile0, sub = sub0;
+        if (i > 0) {
+          item_tile(p, wi.tile, tile, sub);
+          tile_coords(tile, p, tm, tn);
+        }
         // 256-wide half item: one B half-box, into the slot of accumulator half hsel
         // (alternating per item, so consecutive half items double-buffer TMEM)
         const bool half = (NH == 2) && (MC == 1) && sub >= 0;
@@ -592,8 +607,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
         const uint32_t stage_bytes = half ? STAGE_BYTES - B_HALF_BYTES
                                      : flex ? A_BYTES + static_cast<uint32_t>(TB_ROWS) * 128u : STAGE_BYTES;
         if (i == 0) {
-          HG_STAMP2(1);
-          griddep_wait();  // first global access of this role below
+          HG_STAMP2(1);  // (griddep_wait done in the prologue)
           HG_STAMP(2);
         } else if (p.wsync != nullptr && i < p.wsync_items) {
           wave_bar();  // this CTA has issued every load of its items < i

@@ -44,9 +44,9 @@ for f in range(7):
     xs = [r[f] - t0 for r in rows2 if r[f]]
     if xs:
         print(f"{names2[f]:10s} min {min(xs):7d} med {statistics.median(xs):9.0f} max {max(xs):7d}")
-names3 = ["w2_presync", "w5_presync", "t0_postsync", "w2_cpre"]
+names3 = ["w2_presync", "w5_presync", "t0_postsync", "w2_cpre", "w2_tmld0", "w2_staged", "w2_rbar", "w2_summed"]
 rows3 = [v[8 + 4096 + 8 * b: 8 + 4096 + 8 * b + 8] for b in range(256) if v[8 + 8 * b]]
-for f in range(4):
+for f in range(8):
     xs = [r[f] - t0 for r in rows3 if r[f]]
     if xs:
         print(f"{names3[f]:10s} min {min(xs):7d} med {statistics.median(xs):9.0f} max {max(xs):7d}")
