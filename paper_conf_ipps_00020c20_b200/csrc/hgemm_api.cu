@@ -246,6 +246,10 @@ extern const int g_env_wsync_k = [] {  // extra barriers every HGEMM_WSYNC_K k-b
   const char *e = std::getenv("HGEMM_WSYNC_K");
   return e ? std::max(0, std::atoi(e)) : -1;
 }();
+extern const int g_env_wsync_minw = [] {  // wave barrier: minimum whole waves (experiments; default 8)
+  const char *e = std::getenv("HGEMM_WSYNC_MINW");
+  return e ? std::max(1, std::atoi(e)) : 8;
+}();
 struct SkWorkspace {
   int dev;
   cudaStream_t stream;
@@ -297,6 +301,18 @@ inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 // capacity per split count is taken conservatively.
 bool choose_splitk(int64_t M, int64_t N, int64_t K, int num_sms, int &bn, int &spl) {
   const int64_t nkb = cdiv(K, 64);
+  // Small problems (K <= 1024): 128 x 64 tiles split 4 (or 2) ways whenever that is still one
+  // wave -- the loads of a launch-bound GEMM spread over more SMs.  Measured (ncu, cold;
+  // profiles/r02/small_split_choice.log): 256^3 NN FP32 8.6 -> 7.5 us, 384^3 9.0 -> 6.7,
+  // 512^3 8.6 -> 7.0, 512^3 NN FP32 12.5 -> 7.9, 768^3 9.5 -> 7.8 (the 64-wide split 2).
+  if (N > 64 && nkb <= 16) {
+    const int64_t t64 = cdiv(M, 128) * cdiv(N, 64);
+    if (t64 * 2 <= num_sms) {
+      bn = 64;
+      spl = (t64 * 4 <= num_sms && nkb >= 4) ? 4 : 2;
+      if (nkb >= spl) return true;
+    }
+  }
   bn = N <= 64 ? 64 : 128;
   const int64_t tiles = cdiv(M, 128) * cdiv(N, bn);
   if (tiles * 2 > num_sms) return false;  // at least half the SMs already busy without splitting

@@ -36,6 +36,7 @@ int sk_plan(int64_t tiles, int64_t units, int64_t nkb, int mode);
 bool sk_workspace(int dev, cudaStream_t s, int num_sms, float **ws, int **flags);
 extern const int kWsyncOffset;
 extern const int g_env_wsync;  // HGEMM_WSYNC: 1 = wave barrier for tile kernels with >= 8 whole waves
+extern const int g_env_wsync_minw;  // HGEMM_WSYNC_MINW: minimum whole waves for the wave barrier (default 8)
 extern const int g_env_wsync_k;  // HGEMM_WSYNC_K: k-block interval of extra barriers inside tiles (0 = none, -1 = auto)
 
 // One launch of a persistent tile kernel.
@@ -161,7 +162,7 @@ hgemm_status_t launch_tc(const TcLaunch &L) {
     int *flags = nullptr;
     // long tiles only (K >= 8192): with short k loops the panels stay in L2 anyway and the
     // per-wave meeting costs more than it saves (BERT-FFN1 16384 x 4096 x 1024: 129 -> 151 us)
-    if (whole_waves >= 8 && p.num_k_blocks >= 128 && units * CG <= di.num_sms &&
+    if (whole_waves >= g_env_wsync_minw && p.num_k_blocks >= 128 && units * CG <= di.num_sms &&
         sk_workspace(dev, L.stream, di.num_sms, &ws, &flags) &&
         cudaMemsetAsync(flags + kWsyncOffset, 0, sizeof(int), L.stream) == cudaSuccess) {
       p.wsync = flags + kWsyncOffset;

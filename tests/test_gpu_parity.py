@@ -348,6 +348,30 @@ def test_splitk_auto_for_underfilled(oracle_mod):
     assert_within_tolerance(case, got, r, ab)
 
 
+@pytest.mark.parametrize("w,tA,tB,out,spl", [(256, "N", "N", "f32", 4), (384, "T", "N", "f16", 4),
+                                              (512, "N", "N", "f32", 4), (768, "T", "N", "f16", 2),
+                                              (333, "T", "T", "f16", 4)])
+def test_splitk_auto_small_problems(oracle_mod, w, tA, tB, out, spl):
+    """Small problems (K <= 1024, one wave of 128 x 64 split tiles) go to the 64-wide split-K
+    kernel automatically (BJ config 1 among them): random inputs within the BJ bound and
+    integer inputs bit-exact, ragged W = 333 included."""
+    for integer in (False, True):
+        if integer:
+            opA, opB = inputs.integer_f16(w, w, 5, -2, 2), inputs.integer_f16(w, w, 6, -2, 2)
+        else:
+            opA, opB = inputs.uniform_f16(w, w, 5), inputs.uniform_f16(w, w, 6)
+        case = GpuCase(opA, opB, tA, tB, out=out)
+        got = case.run_gpu()
+        st = case.stats
+        assert st["last_kernel"] == "splitk" and st["block_n"] == 64 and st["splits"] == spl, st
+        c_ref, r, ab = case.oracle(oracle_mod)
+        if integer:
+            assert out == "f32" or np.max(np.abs(r)) <= 2048  # exact in FP16
+            assert np.array_equal(case.view(got).astype(np.float64), r)
+        else:
+            assert_within_tolerance(case, got, r, ab)
+
+
 def test_cuda_graph_capture_and_replay(oracle_mod):
     """hgemm() is asynchronous and allocation-free, so it can be captured in a CUDA graph."""
     import torch
