@@ -64,6 +64,7 @@ const int g_env_stream_pre = env_int("HGEMM_STREAM_PRE", 0);    // streaming ker
 const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pair kernel (-DHGEMM_ENABLE_MC)
 const int g_env_group_n = env_int("HGEMM_GROUP_N", 0);        // > 0: raster groups along N
 const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hints
+const int g_env_sk_hm = env_int("HGEMM_SK_HM", 0);            // split-K 64-wide: 64-row tiles (experiments)
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
 const bool g_env_flex = env_int("HGEMM_FLEX", 0) != 0;        // flexible tile widths in the automatic choice
 const int g_env_direct = env_int("HGEMM_EPI_DIRECT", 0);      // 256-wide pair tiles: direct-store epilogue, 7 stages
@@ -299,8 +300,9 @@ inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 // already fills the GPU.  Cluster sizes of 4 and 8 leave some SMs of a GPC
 // unused (148 SMs do not split into 4-CTA clusters evenly), so the
 // capacity per split count is taken conservatively.
-bool choose_splitk(int64_t M, int64_t N, int64_t K, int num_sms, int &bn, int &spl) {
+bool choose_splitk(int64_t M, int64_t N, int64_t K, int num_sms, int &bn, int &spl, bool &hm) {
   const int64_t nkb = cdiv(K, 64);
+  hm = false;
   // Small problems (K <= 1024): 128 x 64 tiles split 4 (or 2) ways whenever that is still one
   // wave -- the loads of a launch-bound GEMM spread over more SMs.  Measured (ncu, cold;
   // profiles/r02/small_split_choice.log): 256^3 NN FP32 8.6 -> 7.5 us, 384^3 9.0 -> 6.7,
@@ -310,6 +312,9 @@ bool choose_splitk(int64_t M, int64_t N, int64_t K, int num_sms, int &bn, int &s
     if (t64 * 2 <= num_sms) {
       bn = 64;
       spl = (t64 * 4 <= num_sms && nkb >= 4) ? 4 : 2;
+      // tiny problems: 64-row tiles (HM) while even those, split 4 ways, fill at most half the
+      // SMs -- 256^3 NN FP32 7.4 -> 6.4 us (profiles/r02/splitk_hm_ab.log)
+      hm = spl == 4 && cdiv(M, 64) * cdiv(N, 64) * 4 <= num_sms / 2;
       if (nkb >= spl) return true;
     }
   }
@@ -690,7 +695,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   // ---------------------------------------------------------- split-K (under-filled shapes)
   {
     int sk_bn = 0, sk_spl = 0;
-    bool use_sk = false;
+    bool use_sk = false, auto_hm = false;
     if (ag || acc16) {
       // the fused all-gather and FP16 accumulation run the persistent tile kernel only
     } else if (cfg.kernel == HGEMM_KERNEL_SPLITK) {
@@ -698,17 +703,23 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
       sk_bn = cfg.block_n ? cfg.block_n : (N <= 64 ? 64 : 128);
       sk_spl = cfg.splits ? cfg.splits : 4;
     } else if (cfg.kernel == HGEMM_KERNEL_AUTO) {
-      use_sk = choose_splitk(M, N, k, di.num_sms, sk_bn, sk_spl);
+      use_sk = choose_splitk(M, N, k, di.num_sms, sk_bn, sk_spl, auto_hm);
     }
+    // 64 x 64 tiles with 64 valid Ak rows (hgemm_splitk.cuh "HM"): twice the tiles, half the splits
+    // (HGEMM_SK_HM=1, experiments: every 64-wide split-K launch, automatic ones with half the splits)
+    const bool hm_ok = use_sk && sk_bn == 64 && g_env_sk_hm > 0;
+    if (hm_ok && cfg.kernel == HGEMM_KERNEL_AUTO && sk_spl > 2 && !auto_hm) sk_spl /= 2;
+    const bool sk_hm = (auto_hm || hm_ok) && (sk_spl == 2 || sk_spl == 4);
     if (use_sk) {
       CUtensorMap ta, tb;
       bool ok;
+      const uint32_t a_box_rows = sk_hm ? 64u : 128u;
       // k-groups of 2 (3-D Ak view, one load of 256 contiguous bytes per Ak row): K-major Ak,
       // K % 64 == 0 and every split's k range a whole number of groups
       const int nkb_all = static_cast<int>(cdiv(k, 64));
       const int sk_kg = (!a_mn && k % 64 == 0 && nkb_all % (2 * sk_spl) == 0 && g_env_sk_kg == 2) ? 2 : 1;
-      if (!a_mn) ok = sk_kg == 2 ? make_map_3d(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 128, 2)
-                                 : make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
+      if (!a_mn) ok = sk_kg == 2 ? make_map_3d(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, a_box_rows, 2)
+                                 : make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, a_box_rows);
       else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
       if (ok) {
         if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, sk_bn);
@@ -719,7 +730,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
       p.M = static_cast<int32_t>(M);
       p.N = static_cast<int32_t>(N);
       p.K = static_cast<int32_t>(k);
-      p.num_m_tiles = static_cast<int32_t>(cdiv(M, 128));
+      p.num_m_tiles = static_cast<int32_t>(cdiv(M, sk_hm ? 64 : 128));
       p.num_n_tiles = static_cast<int32_t>(cdiv(N, sk_bn));
       p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
       p.group_m = p.num_m_tiles;  // tiles in m-fastest order
@@ -729,7 +740,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
       p.D = C;
       p.ldd = ldc;
       p.probe = g_probe.load(std::memory_order_relaxed);
-      const hgemm_status_t st = sk_bn == 64 ? hgi::dispatch_splitk64(sk_spl, a_mn, b_mn, f32, ta, tb, p, dev, stream)
+      const hgemm_status_t st = sk_bn == 64 ? hgi::dispatch_splitk64(sk_spl, a_mn, b_mn, f32, ta, tb, p, dev, stream, sk_hm)
                                             : hgi::dispatch_splitk128(sk_spl, a_mn, b_mn, f32, ta, tb, p, dev, stream);
       if (st == HGEMM_SUCCESS) {
         std::lock_guard<std::mutex> lk(g_mu);

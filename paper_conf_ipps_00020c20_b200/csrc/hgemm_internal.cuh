@@ -58,7 +58,8 @@ hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_m
                                 bool direct = false);
 hgemm_status_t dispatch_tc1(int bn, bool a_mn, bool b_mn, bool f32, const TcLaunch &L);
 hgemm_status_t dispatch_splitk64(int spl, bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta,
-                                 const CUtensorMap &tb, const hg::TcParams &p, int dev, cudaStream_t s);
+                                 const CUtensorMap &tb, const hg::TcParams &p, int dev, cudaStream_t s,
+                                 bool hm = false);
 hgemm_status_t dispatch_splitk128(int spl, bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta,
                                   const CUtensorMap &tb, const hg::TcParams &p, int dev, cudaStream_t s);
 
@@ -234,11 +235,11 @@ hgemm_status_t dispatch_tc_ag(bool a_mn, bool f32, const TcLaunch &L) {
 }
 
 // ----------------------------------------------------------------- split-K launch
-template <int BN, int SPL, bool A_MN, bool B_MN, bool OUT_F32>
+template <int BN, int SPL, bool A_MN, bool B_MN, bool OUT_F32, bool HM = false>
 hgemm_status_t launch_splitk(const CUtensorMap &ta, const CUtensorMap &tb, const hg::TcParams &p, int dev,
                              cudaStream_t stream) {
-  using SH = hg::SkShape<BN, SPL>;
-  auto kern = hg::hgemm_splitk_kernel<BN, SPL, A_MN, B_MN, OUT_F32>;
+  using SH = hg::SkShape<BN, SPL, HM>;
+  auto kern = hg::hgemm_splitk_kernel<BN, SPL, A_MN, B_MN, OUT_F32, HM>;
   static KernInit init;
   std::call_once(init.once[dev], [&] {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SH::SMEM_BYTES);
@@ -265,11 +266,11 @@ hgemm_status_t launch_splitk(const CUtensorMap &ta, const CUtensorMap &tb, const
   return HGEMM_SUCCESS;
 }
 
-template <int BN, int SPL>
+template <int BN, int SPL, bool HM = false>
 hgemm_status_t dispatch_splitk_layout(bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta, const CUtensorMap &tb,
                                       const hg::TcParams &p, int dev, cudaStream_t s) {
 #define HG_SK(AM, BM_, F) \
-  if (a_mn == AM && b_mn == BM_ && f32 == F) return launch_splitk<BN, SPL, AM, BM_, F>(ta, tb, p, dev, s);
+  if (a_mn == AM && b_mn == BM_ && f32 == F) return launch_splitk<BN, SPL, AM, BM_, F, HM>(ta, tb, p, dev, s);
   HG_SK(false, false, false)
   HG_SK(false, false, true)
   HG_SK(false, true, false)

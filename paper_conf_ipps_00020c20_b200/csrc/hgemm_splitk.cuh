@@ -29,11 +29,15 @@
 
 namespace hg {
 
-template <int BN, int S>
+// HM (half M): tiles of 64 valid Ak rows.  The TMA brings 64 rows (8 KB per k-block); the
+// M = 128 MMA reads the next 8 KB of the same stage as rows 64..127 (the next Ak k-block or
+// the stage's Bk), which only feed accumulator lanes 64..127 -- never read.  Twice the tiles for the same K split: the LSTM
+// gates at batch 64 run 64 tiles x 2 splits instead of 32 x 4 (a 2-way reduction).
+template <int BN, int S, bool HM = false>
 struct SkShape {
-  static constexpr int BM = 128;
+  static constexpr int BM = HM ? 64 : 128;                 // valid tile rows
   static constexpr int BK = 64;
-  static constexpr uint32_t A_BYTES = BM * BK * 2;
+  static constexpr uint32_t A_BYTES = BM * BK * 2;         // Ak bytes loaded per k-block
   static constexpr uint32_t B_BYTES = BN * BK * 2;
   static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
   // receive buffer: (S-1) peer slots x 128 rows x BN/S FP32 (peer src lands in slot
@@ -57,11 +61,11 @@ struct SkShape {
 // sender stages in the same layout with S owner slots), the
 // 16-byte chunk index of a row rotated by the row so that consecutive rows
 // (threads) writing or reading the same chunk use different bank groups.
-template <int SLICE>
+template <int SLICE, int ROWS = 128>
 __device__ __forceinline__ uint32_t recv_off_t(uint32_t src, uint32_t row, uint32_t chunk) {
   constexpr uint32_t CH = SLICE / 4;                      // 16-byte chunks per row
   const uint32_t q = (chunk + row) % CH;
-  return (src * 128u + row) * (SLICE * 4u) + q * 16u;
+  return (src * static_cast<uint32_t>(ROWS) + row) * (SLICE * 4u) + q * 16u;
 }
 
 // 16 bytes from registers into a peer CTA's shared memory, completing 16 bytes of
@@ -94,18 +98,18 @@ __device__ __forceinline__ float4 ld_shared_cluster_v4(uint32_t addr) {
   return v;
 }
 
-template <int BN, int S, bool A_MN, bool B_MN, bool OUT_F32>
+template <int BN, int S, bool A_MN, bool B_MN, bool OUT_F32, bool HM = false>
 __global__ void __launch_bounds__(192, 1)
     hgemm_splitk_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                         const TcParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
-  using SH = SkShape<BN, S>;
+  using SH = SkShape<BN, S, HM>;
   constexpr int BM = SH::BM;
   constexpr int BK = SH::BK;
   constexpr int STAGES = SH::STAGES;
   constexpr uint32_t A_BYTES = SH::A_BYTES;
   constexpr uint32_t STAGE_BYTES = SH::STAGE_BYTES;
-  constexpr uint32_t IDESC = make_idesc_f16<BM, BN, A_MN, B_MN>();
+  constexpr uint32_t IDESC = make_idesc_f16<128, BN, A_MN, B_MN>();  // M = 128 (HM: 64 valid rows)
   constexpr uint32_t A_KSTEP = A_MN ? 16 * 128 : 32;
   constexpr uint32_t B_KSTEP = B_MN ? 16 * 128 : 32;
 
@@ -128,7 +132,7 @@ __global__ void __launch_bounds__(192, 1)
   const int kb0 = static_cast<int>((static_cast<int64_t>(p.num_k_blocks) * rank) / S);
   const int kb1 = static_cast<int>((static_cast<int64_t>(p.num_k_blocks) * (rank + 1)) / S);
   const int nkb = kb1 - kb0;
-  auto recv_off = [](uint32_t src, uint32_t row, uint32_t chunk) { return recv_off_t<SH::SLICE>(src, row, chunk); };
+  auto recv_off = [](uint32_t src, uint32_t row, uint32_t chunk) { return recv_off_t<SH::SLICE, BM>(src, row, chunk); };
 
 #ifdef HGEMM_TRACE
 #define SK_TRACE(f)                                                                            \
@@ -223,7 +227,7 @@ __global__ void __launch_bounds__(192, 1)
       mbar_init(rbar, 1);
       // the peers' bulk copies complete their bytes on rbar (possibly before this arrival:
       // the transaction count may run negative until the expectation is registered)
-      mbar_arrive_expect_tx(rbar, (S - 1) * 128u * SH::SLICE * 4u);
+      mbar_arrive_expect_tx(rbar, (S - 1) * static_cast<uint32_t>(BM) * SH::SLICE * 4u);
       fence_mbarrier_init();
     }
     __syncwarp();
@@ -254,7 +258,7 @@ __global__ void __launch_bounds__(192, 1)
     if (warp >= 2 && p.beta != 0.0f) {
       const int row = tm * BM + static_cast<int>((warp & 3u) * 32u + lane);
       const int col0 = tn * BN + static_cast<int>(rank) * SH::SLICE;
-      if (row < p.M && col0 + SH::SLICE <= p.N && (p.ldd & 7) == 0) {
+      if ((warp & 3u) * 32u < static_cast<uint32_t>(BM) && row < p.M && col0 + SH::SLICE <= p.N && (p.ldd & 7) == 0) {
         const uint4 *src = reinterpret_cast<const uint4 *>(static_cast<const __half *>(p.D) +
                                                           static_cast<int64_t>(row) * p.ldd + col0);
 #pragma unroll
@@ -309,9 +313,10 @@ __global__ void __launch_bounds__(192, 1)
     // in the owner's receive layout, then each warp sends its 32 rows of slice o with
     // one bulk copy to owner o's buffer [rank][rows], completing on o's rbar.
     constexpr int SLICE = SH::SLICE;
-    constexpr uint32_t SLAB = 128u * SLICE * 4u;  // one source's slice block: 128 rows x SLICE FP32
+    constexpr uint32_t SLAB = static_cast<uint32_t>(BM) * SLICE * 4u;  // one source's slice block: BM rows x SLICE FP32
     const uint32_t quad = warp & 3u;
     const uint32_t prow = quad * 32u + lane;  // TMEM lane == tile row
+    const bool act = quad * 32u < static_cast<uint32_t>(BM);  // HM: the warps of lanes 64..127 hold no valid rows
     const uint32_t stg = smem_u32(smem);      // staging: [owner][row][SLICE] (recv_off layout)
     float own[SLICE];
     // exp_flags & 64 (experiment): push each 16-B chunk of a peer's slice straight from
@@ -323,6 +328,7 @@ __global__ void __launch_bounds__(192, 1)
     mbar_wait(tfull, 0);
     tc_fence_after();
     if (warp == 2 && lane == 0) SK_TRACE(4);
+    if (act) {
 #pragma unroll
     for (int c = 0; c < BN / 32; ++c) {
       uint32_t v[32];
@@ -352,6 +358,7 @@ __global__ void __launch_bounds__(192, 1)
         }
       }
     }
+    }
     if (warp == 2 && lane == 0) SK_TRACE3(5);
     tc_fence_before();
     if (!direct) {
@@ -359,7 +366,7 @@ __global__ void __launch_bounds__(192, 1)
     __syncwarp();
     cluster_wait();            // every peer's rbar is initialised before we copy into it
     }
-    if (lane == 0 && !direct) {
+    if (lane == 0 && !direct && act) {
       const uint32_t rows_off = quad * 32u * SLICE * 4u;  // this warp's 32 rows in a slice block
 #pragma unroll 1
       for (uint32_t o = 0; o < static_cast<uint32_t>(S); ++o) {
@@ -375,13 +382,13 @@ __global__ void __launch_bounds__(192, 1)
     const int row = tm * BM + static_cast<int>(prow);
     const int col0 = tn * BN + static_cast<int>(rank) * SLICE;
     const uint32_t rbuf = smem_u32(part);
-    if constexpr (S > 1) mbar_wait(rbar, 0);  // the (S-1) peers' slices have landed
+    if (S > 1 && act) mbar_wait(rbar, 0);  // the (S-1) peers' slices have landed
     if (warp == 2 && lane == 0) SK_TRACE3(6);
     float acc[SLICE];
 #pragma unroll
     for (int j = 0; j < SLICE; ++j) acc[j] = 0.0f;
 #pragma unroll
-    for (int src = 0; src < S; ++src) {  // fixed summation order: split 0, 1, ..., S-1
+    for (int src = 0; src < (act ? S : 0); ++src) {  // fixed summation order: split 0, 1, ..., S-1
       if (static_cast<uint32_t>(src) == rank) {
 #pragma unroll
         for (int j = 0; j < SLICE; ++j) acc[j] += own[j];
@@ -398,7 +405,7 @@ __global__ void __launch_bounds__(192, 1)
       }
     }
     if (warp == 2 && lane == 0) SK_TRACE3(7);
-    if (row < p.M) {
+    if (act && row < p.M) {
       const float alpha = p.alpha, beta = p.beta;
       if constexpr (OUT_F32) {
         float *dst = static_cast<float *>(p.D) + static_cast<int64_t>(row) * p.ldd + col0;

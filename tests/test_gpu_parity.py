@@ -350,11 +350,12 @@ def test_splitk_auto_for_underfilled(oracle_mod):
 
 @pytest.mark.parametrize("w,tA,tB,out,spl", [(256, "N", "N", "f32", 4), (384, "T", "N", "f16", 4),
                                               (512, "N", "N", "f32", 4), (768, "T", "N", "f16", 2),
-                                              (333, "T", "T", "f16", 4)])
+                                              (333, "T", "T", "f16", 4), (200, "T", "T", "f16", 4),
+                                              (250, "N", "T", "f32", 4), (130, "T", "N", "f16", 2)])
 def test_splitk_auto_small_problems(oracle_mod, w, tA, tB, out, spl):
     """Small problems (K <= 1024, one wave of 128 x 64 split tiles) go to the 64-wide split-K
-    kernel automatically (BJ config 1 among them): random inputs within the BJ bound and
-    integer inputs bit-exact, ragged W = 333 included."""
+    kernel automatically (BJ config 1 among them; W <= 256 with 64-row "HM" tiles): random
+    inputs within the BJ bound and integer inputs bit-exact, ragged sizes included."""
     for integer in (False, True):
         if integer:
             opA, opB = inputs.integer_f16(w, w, 5, -2, 2), inputs.integer_f16(w, w, 6, -2, 2)
