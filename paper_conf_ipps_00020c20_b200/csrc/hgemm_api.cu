@@ -67,6 +67,7 @@ const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hi
 const int g_env_sk_hm = env_int("HGEMM_SK_HM", 0);            // split-K 64-wide: 64-row tiles (experiments)
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
 const bool g_env_flex = env_int("HGEMM_FLEX", 0) != 0;        // flexible tile widths in the automatic choice
+const int g_env_tc_kg = env_int("HGEMM_TC_KG", 2);            // 256-wide tiles: k-blocks per ring stage (1 or 2)
 const int g_env_direct = env_int("HGEMM_EPI_DIRECT", 0);      // 256-wide pair tiles: direct-store epilogue, 7 stages
 
 bool device_info(int dev, DeviceInfo &out) {
@@ -781,13 +782,29 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   }
 #endif
 
+  // k-group stages (KG = 2: two k-blocks per ring stage, each operand one 3-D TMA box of
+  // 256 contiguous bytes per row): 256-wide tiles, both operands K-major, K % 128 == 0, whole
+  // tiles
+  // Not where the launch would use stream-K (W = 2304 / 2560 / 4608: the 1-k-block stages with
+  // stream-K measured faster) and not for one row of pair tiles (M <= 256: the skinny
+  // HBM-streaming case, where 3 stages of 64 KB keep fewer bytes in flight than 6 of 32 KB);
+  // profiles/r02/tc_kgroup_ab.log.
+  const int64_t kg_tiles = cdiv(M, 256) * cdiv(N, 256);
+  const bool kg2 = g_env_tc_kg == 2 && cg == 2 && bn == 256 && !a_mn && !b_mn && k % 128 == 0 && !tnf && mc == 1 &&
+                   !ag && !acc16 && !(cg == 2 && g_env_direct != 0) && M > 256 &&
+                   sk_plan(kg_tiles, di.num_sms / 2, cdiv(k, 64), skm & 15) < 0;
   CUtensorMap ta, tb;
   bool ok;
-  if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
-  else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
-  if (ok) {
-    if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, b_rows / mc);
-    else ok = make_map(&tb, A, static_cast<uint64_t>(m), static_cast<uint64_t>(k), lda, 64, 64);
+  if (kg2) {
+    ok = make_map_3d(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 128, 2) &&
+         make_map_3d(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, static_cast<uint32_t>(b_rows), 2);
+  } else {
+    if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
+    else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
+    if (ok) {
+      if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, b_rows / mc);
+      else ok = make_map(&tb, A, static_cast<uint64_t>(m), static_cast<uint64_t>(k), lda, 64, 64);
+    }
   }
   // D = C^T row-major (N = m contiguous), stored in 32-row x 128-B swizzled boxes
   CUtensorMap td;
@@ -839,14 +856,15 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   bool sk_used = false;
   const hgi::TcLaunch L = {&ta, &tb, &td, &p, dev, &di, cfg.max_ctas, skm_eff, &sk_used, stream};
   hgemm_status_t st;
-  if (cg == 2 && bn == 512) st = hgi::dispatch_tc512(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
+  if (kg2) st = hgi::dispatch_tc256_kg2(cg, f32, L);
+  else if (cg == 2 && bn == 512) st = hgi::dispatch_tc512(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
   else if (cg == 2)
     st = hgi::dispatch_tc256x2(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L, g_env_direct != 0 && !tnf);
   else st = hgi::dispatch_tc1(bn, a_mn, b_mn, f32, L);
   if (st == HGEMM_SUCCESS) {
     std::lock_guard<std::mutex> lk(g_mu);
-    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, 0, sk_used ? 2 : 1,
-              t_half_used ? 2 : 1, tnf};
+    g_last = {cg == 2 ? HGEMM_KERNEL_TC_2SM : HGEMM_KERNEL_TC_1SM, bn, p.group_m, cfg.max_ctas, kg2 ? 2 : 0,
+              sk_used ? 2 : 1, t_half_used ? 2 : 1, tnf};  // splits: k-blocks per ring stage when 2 (KG)
   }
   return st;
 }

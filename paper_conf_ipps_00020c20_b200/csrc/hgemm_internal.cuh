@@ -57,6 +57,9 @@ hgemm_status_t dispatch_tc512(int mc, bool ag, bool acc16, bool a_mn, bool b_mn,
 hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_mn, bool f32, const TcLaunch &L,
                                 bool direct = false);
 hgemm_status_t dispatch_tc1(int bn, bool a_mn, bool b_mn, bool f32, const TcLaunch &L);
+// 256-wide CTA-pair tiles with k-group stages (KG = 2): TN layout,
+// K % 128 == 0, whole tiles; tensor maps are the 3-D k-group views (box {64, rows, 2})
+hgemm_status_t dispatch_tc256_kg2(int cg, bool f32, const TcLaunch &L);
 hgemm_status_t dispatch_splitk64(int spl, bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta,
                                  const CUtensorMap &tb, const hg::TcParams &p, int dev, cudaStream_t s,
                                  bool hm = false);
@@ -73,16 +76,17 @@ struct KernInit {
   int max_clusters[kMaxDevices] = {};
 };
 
-template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC, bool AG, bool ACC16, bool DIRECT = false>
+template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC, bool AG, bool ACC16, bool DIRECT = false,
+          int KG = 1>
 hgemm_status_t launch_tc(const TcLaunch &L) {
-  using S = hg::TcShape<BN, CG, OUT_F32, DIRECT>;
+  using S = hg::TcShape<BN, CG, OUT_F32, DIRECT, KG>;
   constexpr int THREADS = S::THREADS + (AG ? 32 : 0);  // + the all-gather copy warp
   const int dev = L.dev;
   const DeviceInfo &di = *L.di;
   const hg::TcParams &p0 = *L.p;
   const int ht_mode = L.sk_mode >> 4;  // hgemm_config_t::half_tail, packed above the stream-K mode
   const int sk_mode = L.sk_mode & 15;
-  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC, AG, ACC16, DIRECT>;
+  auto kern = hg::hgemm_tc_kernel<BN, CG, A_MN, B_MN, OUT_F32, MC, AG, ACC16, DIRECT, KG>;
   static KernInit init;
   std::call_once(init.once[dev], [&] {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, S::SMEM_BYTES);
@@ -134,7 +138,8 @@ hgemm_status_t launch_tc(const TcLaunch &L) {
   }
   t_half_used = half_tail;
   if (MC == 1 && !AG && !ACC16 && !half_tail) {
-    const int dp = sk_plan(tiles, units, p.num_k_blocks, sk_mode);
+    // k-group stages (KG = 2) run whole tiles only (work items of an even number of k-blocks)
+    const int dp = sk_plan(tiles, units, p.num_k_blocks, KG == 2 ? 1 : sk_mode);
     float *ws = nullptr;
     int *flags = nullptr;
     if (dp >= 0 && units * CG * MC <= di.num_sms && sk_workspace(dev, L.stream, di.num_sms, &ws, &flags)) {

@@ -237,7 +237,11 @@ __device__ __forceinline__ uint32_t pack_half2(float a, float b) {
   return *reinterpret_cast<uint32_t *>(&h);
 }
 
-template <int BN, int CG, bool OUT_F32, bool EPI_DIRECT = false>
+// KG (k-group): a ring stage holds KG consecutive k-blocks, each operand brought by ONE 3-D
+// TMA load of KG x 128 contiguous bytes per row (DESIGN.md "k-group loads in the tile
+// kernel"): the TMA engine's throughput per SM is set by box rows, not bytes
+// (profiles/r02/l2_ingest_study.log), so 256-B rows double the bytes it delivers per SM.
+template <int BN, int CG, bool OUT_F32, bool EPI_DIRECT = false, int KG = 1>
 struct TcShape {
   static constexpr int BM = 128;                       // rows per CTA (TMEM lanes)
   static constexpr int BK = 64;                        // FP16 per 128-B swizzle atom
@@ -247,7 +251,7 @@ struct TcShape {
   static constexpr uint32_t A_BYTES = BM * BK * 2;
   static constexpr uint32_t B_HALF_BYTES = B_ROWS * BK * 2;
   static constexpr uint32_t B_BYTES = NH * B_HALF_BYTES;
-  static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr uint32_t STAGE_BYTES = KG * (A_BYTES + B_BYTES);  // one ring stage: KG k-blocks
   static constexpr int ACC = (2 * BN <= 512) ? 2 : 1;  // accumulator buffers in TMEM
   static constexpr uint32_t TMEM_COLS = (ACC * BN <= 256) ? 256 : 512;
   static constexpr int EPI_COLS = OUT_F32 ? 32 : 64;   // one 128-B staging row per thread
@@ -462,12 +466,14 @@ __device__ __forceinline__ void ag_copy_warp(const TcParams &p, uint32_t lane) {
 }
 
 template <int BN, int CG, bool A_MN, bool B_MN, bool OUT_F32, int MC = 1, bool AG = false, bool ACC16 = false,
-          bool EPI_DIRECT = false>
-__global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS + (AG ? 32 : 0), 1)
+          bool EPI_DIRECT = false, int KG = 1>
+__global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT, KG>::THREADS + (AG ? 32 : 0), 1)
     hgemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmD, const TcParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
-  using S = TcShape<BN, CG, OUT_F32, EPI_DIRECT>;
+  using S = TcShape<BN, CG, OUT_F32, EPI_DIRECT, KG>;
+  static_assert(KG == 1 || (KG == 2 && S::NH == 1 && !A_MN && !B_MN && MC == 1 && !AG),
+                "k-group stages: one accumulator half, K-major operands, whole tiles");
   constexpr int BM = S::BM;
   constexpr int BK = S::BK;
   constexpr int UMMA_N = S::UMMA_N;
@@ -627,7 +633,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
           }
           fence_proxy_async_global();  // the copy warps' generic stores -> this CTA's TMA (async proxy) reads
         }
-        for (int kb = wi.kb0; kb < wi.kb1; ++kb) {
+        for (int kb = wi.kb0; kb < wi.kb1; kb += KG) {
           if (p.wsync_kint > 0 && p.wsync != nullptr && i < p.wsync_items && kb > wi.kb0 &&
               (kb - wi.kb0) % p.wsync_kint == 0)
             wave_bar();  // k-block alignment inside the tile (experiment, HGEMM_WSYNC_K)
@@ -638,7 +644,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
           if (i == 0 && kb == wi.kb0) HG_STAMP2(2);
 #endif
           const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES);
-          const uint32_t sb = sa + A_BYTES;
+          const uint32_t sb = sa + KG * A_BYTES;
           uint32_t fb;
           if constexpr (CG == 1) {
             mbar_arrive_expect_tx(&full[stage], stage_bytes);
@@ -651,7 +657,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
 #ifdef HGEMM_TRACE
           if (i == 0 && kb == wi.kb0) HG_STAMP2(3);
 #endif
-          if constexpr (!A_MN) {
+          if constexpr (!A_MN && KG == 2) {  // k-blocks kb, kb+1 of the Ak rows: one 3-D box
+            if constexpr (CG == 1) tma_load_3d(&tmA, sa, fb, 0, a_row, kb);
+            else tma_load_3d_pair(&tmA, sa, fb, 0, a_row, kb);
+          } else if constexpr (!A_MN) {
             if constexpr (CG == 1) tma_load_2d(&tmA, sa, fb, k0, a_row, pol_a);
             else tma_load_2d_pair(&tmA, sa, fb, k0, a_row, pol_a);
 #ifdef HGEMM_TRACE
@@ -668,7 +677,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
           for (int hh = 0; hh < NH; ++hh) {
             if (half && hh > 0) break;
             const int h = half ? hsel : hh;
-            const uint32_t sbh = sb + h * B_HALF_BYTES;
+            const uint32_t sbh = sb + h * KG * B_HALF_BYTES;
             const int b_row = b_row0 + (half ? sub : h) * UMMA_N;
             if constexpr (MC == 2) {
               // this pair's share of the half-box, delivered to the same CTA position of both pairs
@@ -680,7 +689,10 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
                 tma_load_2d_pair_mc(&tmB, sbh + pair * 8192u, fb, b_row + 64 * static_cast<int>(pair), k0, mc_mask);
               continue;
             }
-            if constexpr (!B_MN) {
+            if constexpr (!B_MN && KG == 2) {
+              if constexpr (CG == 1) tma_load_3d(&tmB, sbh, fb, 0, b_row, kb);
+              else tma_load_3d_pair(&tmB, sbh, fb, 0, b_row, kb);
+            } else if constexpr (!B_MN) {
               if constexpr (CG == 1) tma_load_2d(&tmB, sbh, fb, k0, b_row, pol_b);
               else tma_load_2d_pair(&tmB, sbh, fb, k0, b_row, pol_b);
             } else {
@@ -697,7 +709,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }
           // the first ring's worth of operand loads is queued: the epilogue's C loads
           // (beta != 0) may follow without delaying the start of the mainloop
-          if (!cgo_sent && (i > 0 || kb + 1 - wi.kb0 >= STAGES || kb + 1 == wi.kb1)) {
+          if (!cgo_sent && (i > 0 || kb + KG - wi.kb0 >= STAGES * KG || kb + KG >= wi.kb1)) {
             mbar_arrive(cgo);
             cgo_sent = true;
           }
@@ -722,12 +734,15 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
       constexpr int MAX_LEAD = STAGES - 1;
       uint32_t stage = 0, phase = 0;
       int it = 0;
-      auto issue_half = [&](uint32_t st, int h, int kbl, uint32_t d_tmem) {
-        const uint32_t sa = smem_u32(smem + st * STAGE_BYTES);
+      // k-block jj of ring stage st (KG k-blocks per stage: [KG Ak][KG Bk per half])
+      auto issue_half = [&](uint32_t st, int h, int kbl, uint32_t d_tmem, int jj = 0) {
+        const uint32_t s0 = smem_u32(smem + st * STAGE_BYTES);
+        const uint32_t sa = s0 + jj * A_BYTES;
+        const uint32_t sbj = s0 + KG * A_BYTES + h * KG * B_HALF_BYTES + jj * B_HALF_BYTES;
 #pragma unroll
         for (int k = 0; k < BK / 16; ++k) {
           const uint32_t a_addr = sa + k * A_KSTEP;
-          const uint32_t b_addr = sa + A_BYTES + h * B_HALF_BYTES + k * B_KSTEP;
+          const uint32_t b_addr = sbj + k * B_KSTEP;
           const uint64_t ad = A_MN ? sdesc_mn_sw128(a_addr, 8192) : sdesc_k_sw128(a_addr);
           const uint64_t bd = B_MN ? sdesc_mn_sw128(b_addr, 8192) : sdesc_k_sw128(b_addr);
           umma_f16<CG>(d_tmem + h * UMMA_N, ad, bd, idesc, (kbl | k) != 0 ? 1u : 0u);
@@ -805,7 +820,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
 #ifdef HGEMM_TRACE
         long long full_wait = 0;
 #endif
-        for (int kb = 0; kb < nkb; ++kb) {
+        for (int kb = 0; kb < nkb; kb += KG) {
 #ifdef HGEMM_TRACE
           const long long tw0 = clock64();
 #endif
@@ -846,7 +861,8 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT>::THREADS 
               if (h1_ready) flush_h1(min(kb + 1, h1_limit));
             }
           } else {
-            issue_half(stage, 0, kb, d_tmem);
+#pragma unroll
+            for (int jj = 0; jj < KG; ++jj) issue_half(stage, 0, kb + jj, d_tmem, jj);
             umma_commit_mask<CG>(&empty[stage], empty_mask);  // frees the smem stage once these MMAs retire
           }
           if (++stage == STAGES) { stage = 0; phase ^= 1u; }

@@ -151,6 +151,15 @@ __device__ __forceinline__ void tma_load_2d(const CUtensorMap *m, uint32_t dst, 
 }
 // 3D tile load (k-block-grouped views: dims {64, rows, k/64}, box {64, rows, G}),
 // completing on a local barrier.
+// 3-D box for the CTA pair (cta_group::2): the bytes complete on the leader CTA's mbarrier.
+__device__ __forceinline__ void tma_load_3d_pair(const CUtensorMap *m, uint32_t dst, uint32_t bar_cluster, int32_t c0,
+                                                 int32_t c1, int32_t c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(bar_cluster), "r"(c0), "r"(c1), "r"(c2)
+      : "memory");
+}
 __device__ __forceinline__ void tma_load_3d(const CUtensorMap *m, uint32_t dst, uint32_t bar, int32_t c0,
                                             int32_t c1, int32_t c2) {
   asm volatile(

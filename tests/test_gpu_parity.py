@@ -373,6 +373,44 @@ def test_splitk_auto_small_problems(oracle_mod, w, tA, tB, out, spl):
             assert_within_tolerance(case, got, r, ab)
 
 
+@pytest.mark.parametrize("m,n,k", [(520, 600, 1024), (300, 1100, 384), (1000, 700, 2048)])
+@pytest.mark.parametrize("out", ["f16", "f32"])
+@pytest.mark.parametrize("beta", [0.0, 1.0])
+def test_tc_kgroup_stages(oracle_mod, m, n, k, out, beta):
+    """256-wide CTA-pair tiles with two k-blocks per ring stage (3-D TMA boxes; layout TN,
+    k % 128 == 0, stream-K off): random inputs within the BJ bound, integer inputs bit-exact,
+    ragged m / n."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("tc2", block_n=256, stream_k=1)
+    for integer in (False, True):
+        if integer:
+            opA, opB = inputs.integer_f16(m, k, 21, -2, 2), inputs.integer_f16(k, n, 22, -2, 2)
+            C = inputs.integer_f16(m, n, 23, -16, 16)
+        else:
+            opA, opB, C = inputs.uniform_f16(m, k, 21), inputs.uniform_f16(k, n, 22), inputs.uniform_f16(m, n, 23)
+        case = GpuCase(opA, opB, "T", "N", 1.0, beta, C=C, out=out)
+        got = case.run_gpu()
+        assert case.stats["last_kernel"] == "tc2" and case.stats["block_n"] == 256, case.stats
+        assert case.stats["splits"] == 2, case.stats   # k-group stages
+        c_ref, r, ab = case.oracle(oracle_mod)
+        if integer:
+            assert out == "f32" or np.max(np.abs(r)) <= 2048
+            assert np.array_equal(case.view(got).astype(np.float64), r)
+        else:
+            assert_within_tolerance(case, got, r, ab)
+
+
+def test_tc_kgroup_accumulator_width(oracle_mod):
+    """k-group stages keep the FP32 accumulator: k/16 - 2 exactly (512 x 512, k = 4096, TN)."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("tc2", block_n=256, stream_k=1)
+    a, b, expect = inputs.accumulator_width_case(512, 512, 4096)
+    case = GpuCase(a, b, "T", "N", out="f32")
+    got = case.view(case.run_gpu())
+    assert case.stats["splits"] == 2, case.stats
+    assert np.all(got == expect), np.unique(got)[:5]
+
+
 def test_cuda_graph_capture_and_replay(oracle_mod):
     """hgemm() is asynchronous and allocation-free, so it can be captured in a CUDA graph."""
     import torch
