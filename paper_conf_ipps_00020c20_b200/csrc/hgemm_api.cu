@@ -67,6 +67,7 @@ const int g_env_l2_hint = env_int("HGEMM_L2_HINT", 0);        // TMA L2 cache hi
 const int g_env_sk_hm = env_int("HGEMM_SK_HM", 0);            // split-K 64-wide: 64-row tiles (experiments)
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
 const bool g_env_flex = env_int("HGEMM_FLEX", 0) != 0;        // flexible tile widths in the automatic choice
+const int g_env_stream_a3d = env_int("HGEMM_STREAM_A3D", 1);  // streaming kernel: Ak through the 3-D k-group view
 const int g_env_tc_kg = env_int("HGEMM_TC_KG", 2);            // 256-wide tiles: k-blocks per ring stage (1 or 2)
 const int g_env_direct = env_int("HGEMM_EPI_DIRECT", 0);      // 256-wide pair tiles: direct-store epilogue, 7 stages
 
@@ -417,9 +418,12 @@ hgemm_status_t run_stream(const void *R, int64_t ldr, int64_t Ms, const void *S,
   // 8 KB past the 64 real Ak rows: the next k-block, the stage's Bk or the pad)
   const uint32_t a_rows = (Ms <= 64) ? 64u : 128u;
   CUtensorMap ta, tb;
-  bool ok = make_map(&ta, R, static_cast<uint64_t>(k), static_cast<uint64_t>(Ms), ldr, 64, a_rows);
   const uint32_t a_bytes = a_rows == 64 ? 8192u : static_cast<uint32_t>(mt) * 16384u;
   const int kg = stream_kgroup(k, a_bytes, cw);
+  // Ak through the 3-D k-group view as well (one row request per 256 B; MT == 1, G == 2)
+  const int a3d = (mt == 1 && kg == 2 && g_env_stream_a3d) ? 1 : 0;
+  bool ok = a3d ? make_map_3d(&ta, R, static_cast<uint64_t>(k), static_cast<uint64_t>(Ms), ldr, a_rows, 2)
+                : make_map(&ta, R, static_cast<uint64_t>(k), static_cast<uint64_t>(Ms), ldr, 64, a_rows);
   if (ok) ok = kg > 1 ? make_map_3d(&tb, S, static_cast<uint64_t>(k), static_cast<uint64_t>(Ns), lds, cw, kg)
                       : make_map(&tb, S, static_cast<uint64_t>(k), static_cast<uint64_t>(Ns), lds, 64, cw);
   if (!ok) return HGEMM_ERR_CUDA;
@@ -433,6 +437,7 @@ hgemm_status_t run_stream(const void *R, int64_t ldr, int64_t Ms, const void *S,
   p.a_bytes = a_bytes;
   p.kg = kg;
   p.b3d = kg > 1 ? 1 : 0;
+  p.a3d = a3d;
   p.stage_bytes = static_cast<uint32_t>(kg) * (a_bytes + static_cast<uint32_t>(cw) * 128u);
   p.stages = static_cast<int32_t>(std::min<uint32_t>(
       hg::kStreamMaxStages, (hg::kStreamSmemBytes - 1536u - (a_rows == 64 ? 8192u : 0u)) / p.stage_bytes));

@@ -58,6 +58,10 @@ struct StreamParams {
   // 26.6 us instead of 28.7 us for 128 MiB at G >= 2 (5.04 vs 4.67 TB/s).
   int32_t b3d;
   int32_t pre;            // stage loads issued before the CTA barrier (1 .. stages)
+  // 1: tmA is the 3-D k-group view of Ak too (MT == 1, kg == 2): the stage's two Ak k-blocks
+  // (64 or 128 rows each) come from ONE load of 256 contiguous bytes per row (the TMA engine
+  // is limited by row requests)
+  int32_t a3d;
 };
 
 #ifdef HGEMM_TRACE
@@ -139,9 +143,13 @@ __global__ void __launch_bounds__(192, 1)
       const uint32_t sa = smem_u32(smem + pstage * stage_bytes);
       mbar_arrive_expect_tx(&full[pstage], stage_bytes);
       const uint32_t fb = smem_u32(&full[pstage]);
-      for (int j = 0; j < kg; ++j) {
+      if (MT == 1 && p.a3d) {
+        tma_load_3d(&tmA, sa, fb, 0, 0, kb0);
+      } else {
+        for (int j = 0; j < kg; ++j) {
 #pragma unroll
-        for (int t = 0; t < MT; ++t) tma_load_2d(&tmA, sa + j * a_bytes + t * A_SUB, fb, (kb0 + j) * 64, t * 128, 0);
+          for (int t = 0; t < MT; ++t) tma_load_2d(&tmA, sa + j * a_bytes + t * A_SUB, fb, (kb0 + j) * 64, t * 128, 0);
+        }
       }
       if (p.b3d) tma_load_3d(&tmB, sa + b_off, fb, 0, pch * cw, kb0);
       else tma_load_2d(&tmB, sa + b_off, fb, kb0 * 64, pch * cw, 0);
