@@ -59,6 +59,7 @@ const int g_env_stream_rot = env_int("HGEMM_STREAM_ROT", 1);  // streaming kerne
 const int g_env_stream_stages = env_int("HGEMM_STREAM_STAGES", 0);  // experiments: cap on the streaming ring depth
 const int g_env_stream_g = env_int("HGEMM_STREAM_G", -1);  // streaming kernel k-blocks per stage (3-D Bk map); -1: auto
 const int g_env_stream_mmax = env_int("HGEMM_STREAM_MMAX", 128);  // largest M (= n) the streaming kernel is chosen for
+const int g_env_sk_b3d = env_int("HGEMM_SK_B3D", 1);          // split-K: op(A) through the 3-D k-group view
 const int g_env_sk_kg = env_int("HGEMM_SK_KG", 2);            // split-K kernel k-blocks per stage (1 or 2)
 const int g_env_stream_pre = env_int("HGEMM_STREAM_PRE", 0);    // streaming kernel stage loads before the CTA barrier (0: all)
 const int g_env_mc = env_int("HGEMM_MC", 1);                  // 2: multicast pair kernel (-DHGEMM_ENABLE_MC)
@@ -724,11 +725,15 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
       // K % 64 == 0 and every split's k range a whole number of groups
       const int nkb_all = static_cast<int>(cdiv(k, 64));
       const int sk_kg = (!a_mn && k % 64 == 0 && nkb_all % (2 * sk_spl) == 0 && g_env_sk_kg == 2) ? 2 : 1;
+      // op(A) (Bk) through the 3-D k-group view too: one row request per 256 B (DESIGN.md
+      // "k-group loads in the tile kernel")
+      const int sk_b3d = (sk_kg == 2 && !b_mn && g_env_sk_b3d) ? 1 : 0;
       if (!a_mn) ok = sk_kg == 2 ? make_map_3d(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, a_box_rows, 2)
                                  : make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, a_box_rows);
       else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
       if (ok) {
-        if (!b_mn) ok = make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, sk_bn);
+        if (!b_mn) ok = sk_b3d ? make_map_3d(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, sk_bn, 2)
+                               : make_map(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, 64, sk_bn);
         else ok = make_map(&tb, A, static_cast<uint64_t>(m), static_cast<uint64_t>(k), lda, 64, 64);
       }
       if (!ok) return HGEMM_ERR_CUDA;
@@ -741,6 +746,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
       p.num_k_blocks = static_cast<int32_t>(cdiv(k, 64));
       p.group_m = p.num_m_tiles;  // tiles in m-fastest order
       p.sk_kg = sk_kg;
+      p.sk_b3d = sk_b3d;
       p.alpha = alpha;
       p.beta = beta;
       p.D = C;

@@ -188,7 +188,9 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll
         for (int q = 0; q < BM / 64; ++q) tma_load_2d(&tmA, sa + q * 8192, fb, a_row + 64 * q, k0, 0);
       }
-      for (int j = 0; j < kg; ++j) {
+      if (!B_MN && kg == 2 && p.sk_b3d) {  // both Bk k-blocks of the stage: one 3-D box, 256 B per row
+        tma_load_3d(&tmB, sb, fb, 0, b_row, pkb);
+      } else for (int j = 0; j < kg; ++j) {
         if constexpr (!B_MN) {
           tma_load_2d(&tmB, sb + j * SH::B_BYTES, fb, k0 + j * BK, b_row, 0);
         } else {

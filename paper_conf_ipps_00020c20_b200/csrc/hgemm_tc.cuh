@@ -98,6 +98,7 @@ struct TcParams {
                       // 4 = wait for store completion before exit, 8 = no PDL trigger, 16 = no cluster
                       // attribute for 1-CTA launches (host side)
   int32_t sk_kg;      // split-K kernel: k-blocks per ring stage (1, or 2 with tmA the 3-D k-group view)
+  int32_t sk_b3d;     // split-K kernel, sk_kg == 2: tmB is the 3-D k-group view too (K-major op(A))
 };
 
 // One unit of work of a cluster: k-blocks [kb0, kb1) of cluster tile `tile`.
