@@ -64,8 +64,33 @@ struct SkShape {
 template <int SLICE, int ROWS = 128>
 __device__ __forceinline__ uint32_t recv_off_t(uint32_t src, uint32_t row, uint32_t chunk) {
   constexpr uint32_t CH = SLICE / 4;                      // 16-byte chunks per row
-  const uint32_t q = (chunk + row) % CH;
+  // 16-B accesses go to shared memory in phases of 8 lanes (rows): the 8 rows of a phase
+  // must cover the 8 16-B bank groups.  Rows are CH chunks apart, so consecutive rows repeat
+  // the bank group every 8/CH rows when CH < 8: rotate by row / (8/CH) then.
+  constexpr uint32_t D = CH >= 8 ? 1u : 8u / CH;
+  const uint32_t q = (chunk + row / D) % CH;
   return (src * static_cast<uint32_t>(ROWS) + row) * (SLICE * 4u) + q * 16u;
+}
+
+// NC consecutive TMEM columns of this thread's lane (32x32b shape), NC = 8, 16, 32 or 64.
+template <int NC>
+__device__ __forceinline__ void sk_tmem_ld(uint32_t taddr, uint32_t *r) {
+  if constexpr (NC == 8) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+                 : "r"(taddr));
+  } else if constexpr (NC == 16) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
+        "{%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr));
+  } else {
+#pragma unroll
+    for (int c = 0; c < NC / 32; ++c)
+      tmem_ld_32x32b_x32(taddr + c * 32, *reinterpret_cast<uint32_t(*)[32]>(r + 32 * c));
+  }
 }
 
 // 16 bytes from registers into a peer CTA's shared memory, completing 16 bytes of
@@ -330,36 +355,46 @@ __global__ void __launch_bounds__(192, 1)
     mbar_wait(tfull, 0);
     tc_fence_after();
     if (warp == 2 && lane == 0) SK_TRACE(4);
-    if (act) {
+    // Slice t of this row is owned by CTA (rank + t) % S; t = 0 is this CTA's own slice.  The
+    // TMEM column offset of a slice is a runtime value (the rank), so each slice is one TMEM
+    // load and its chunk offsets in the receive layout are per-thread constants: no per-chunk
+    // branching on the owner (the unrolled per-column version executed ~500 instructions per
+    // thread here).
+    uint32_t qoff[SLICE / 4];  // this row's 16-B chunk q inside a slice block (recv_off swizzle)
 #pragma unroll
-    for (int c = 0; c < BN / 32; ++c) {
-      uint32_t v[32];
+    for (int q = 0; q < SLICE / 4; ++q) qoff[q] = recv_off(0u, prow, static_cast<uint32_t>(q));
+    if (act) {
+      uint32_t w[S][SLICE];
       if (nkb > 0) {
-        tmem_ld_32x32b_x32(tmem_base + ((quad * 32u) << 16) + c * 32, v);
+#pragma unroll
+        for (int t = 0; t < S; ++t)
+          sk_tmem_ld<SLICE>(tmem_base + ((quad * 32u) << 16) + ((rank + t) & (S - 1)) * SLICE, w[t]);
         tmem_ld_wait();
-        if (c == 0 && warp == 2 && lane == 0) SK_TRACE3(4);
+        if (warp == 2 && lane == 0) SK_TRACE3(4);
       } else {
 #pragma unroll
-        for (int j = 0; j < 32; ++j) v[j] = 0u;
+        for (int t = 0; t < S; ++t)
+#pragma unroll
+          for (int j = 0; j < SLICE; ++j) w[t][j] = 0u;
       }
 #pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const int colq = c * 32 + 4 * q;                  // first of these 4 tile columns
-        const uint32_t owner = static_cast<uint32_t>(colq / SLICE);
-        const uint32_t within = static_cast<uint32_t>(colq % SLICE) / 4;  // 16-B chunk in the slice
-        if (owner == rank) {
+      for (int j = 0; j < SLICE; ++j) own[j] = __uint_as_float(w[0][j]);
 #pragma unroll
-          for (int e = 0; e < 4; ++e) own[(colq % SLICE) + e] = __uint_as_float(v[4 * q + e]);
-        } else if (direct) {
+      for (int t = 1; t < S; ++t) {
+        const uint32_t owner = (rank + t) & (S - 1);
+        if (direct) {
           const uint32_t slot = rank < owner ? rank : rank - 1u;
-          st_async_v4(mapa_shared(part_u32 + recv_off(slot, prow, within), owner), v[4 * q], v[4 * q + 1],
-                      v[4 * q + 2], v[4 * q + 3], mapa_shared(rbar_u32, owner));
+          const uint32_t rbase = mapa_shared(part_u32 + slot * SLAB, owner), rb = mapa_shared(rbar_u32, owner);
+#pragma unroll
+          for (int q = 0; q < SLICE / 4; ++q)
+            st_async_v4(rbase + qoff[q], w[t][4 * q], w[t][4 * q + 1], w[t][4 * q + 2], w[t][4 * q + 3], rb);
         } else {
-          st_shared_v4(stg + owner * SLAB + recv_off(0u, prow, within), v[4 * q], v[4 * q + 1], v[4 * q + 2],
-                       v[4 * q + 3]);
+          const uint32_t base = stg + owner * SLAB;
+#pragma unroll
+          for (int q = 0; q < SLICE / 4; ++q)
+            st_shared_v4(base + qoff[q], w[t][4 * q], w[t][4 * q + 1], w[t][4 * q + 2], w[t][4 * q + 3]);
         }
       }
-    }
     }
     if (warp == 2 && lane == 0) SK_TRACE3(5);
     tc_fence_before();
@@ -396,10 +431,11 @@ __global__ void __launch_bounds__(192, 1)
         for (int j = 0; j < SLICE; ++j) acc[j] += own[j];
         continue;
       }
+      const uint32_t slot = static_cast<uint32_t>(src) < rank ? static_cast<uint32_t>(src) : static_cast<uint32_t>(src) - 1u;
+      const uint32_t sbase = rbuf + slot * SLAB;
 #pragma unroll
       for (int q = 0; q < SLICE / 4; ++q) {
-        const uint32_t slot = static_cast<uint32_t>(src) < rank ? static_cast<uint32_t>(src) : static_cast<uint32_t>(src) - 1u;
-        const float4 v = ld_shared_f4(rbuf + recv_off(slot, prow, q));
+        const float4 v = ld_shared_f4(sbase + qoff[q]);
         acc[4 * q + 0] += v.x;
         acc[4 * q + 1] += v.y;
         acc[4 * q + 2] += v.z;
