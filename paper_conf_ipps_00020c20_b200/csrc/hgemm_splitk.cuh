@@ -350,7 +350,9 @@ __global__ void __launch_bounds__(192, 1)
     // registers into the owner's receive buffer (st.async, completing on its rbar) instead
     // of staging the slices locally and sending them with bulk copies
     const bool direct = (p.exp_flags & 64) != 0;
-    if (direct) cluster_wait();  // every peer's rbar is initialised before we store into it
+    // Every peer's rbar is initialised before we copy / store into it: the cluster barrier's
+    // wait phase, taken here while the mainloop runs (all CTAs arrived in their prologues).
+    cluster_wait();
     const uint32_t part_u32 = smem_u32(part), rbar_u32 = smem_u32(rbar);
     mbar_wait(tfull, 0);
     tc_fence_after();
@@ -399,9 +401,8 @@ __global__ void __launch_bounds__(192, 1)
     if (warp == 2 && lane == 0) SK_TRACE3(5);
     tc_fence_before();
     if (!direct) {
-    fence_proxy_async_smem();  // the staged slices -> the bulk copies (async proxy)
-    __syncwarp();
-    cluster_wait();            // every peer's rbar is initialised before we copy into it
+      fence_proxy_async_smem();  // the staged slices -> the bulk copies (async proxy)
+      __syncwarp();
     }
     if (lane == 0 && !direct && act) {
       const uint32_t rows_off = quad * 32u * SLICE * 4u;  // this warp's 32 rows in a slice block

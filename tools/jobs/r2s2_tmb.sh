@@ -1,7 +1,7 @@
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "splitk or small_problems or lstm" > gpurun_out/s2_tmb_tests.log 2>&1; tail -2 gpurun_out/s2_tmb_tests.log
 for v in new base; do
-  if [ $v = base ]; then export HGEMM_LIB=ab_libs/base8.so; else unset HGEMM_LIB; fi
+  if [ $v = base ]; then export HGEMM_LIB=ab_libs/base9.so; else unset HGEMM_LIB; fi
   for wl in cfg3_lstm_b64 cfg3_lstm_b256 cfg1_256_NN_f32; do
     python tools/ncu_configs.py $wl > /dev/null 2>&1
     ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/tmb_${v}_$wl.csv \
