@@ -801,7 +801,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   // HBM-streaming case, where 3 stages of 64 KB keep fewer bytes in flight than 6 of 32 KB);
   // profiles/r02/tc_kgroup_ab.log.
   const int64_t kg_tiles = cdiv(M, 256) * cdiv(N, 256);
-  const bool kg2 = g_env_tc_kg == 2 && cg == 2 && bn == 256 && !a_mn && !b_mn && k % 128 == 0 && !tnf && mc == 1 &&
+  const bool kg2 = g_env_tc_kg == 2 && cg == 2 && bn == 256 && !a_mn && !b_mn && k % 128 == 0 && !tnf &&
                    !ag && !acc16 && !(cg == 2 && g_env_direct != 0) && M > 256 &&
                    sk_plan(kg_tiles, di.num_sms / 2, cdiv(k, 64), skm & 15) < 0;
   CUtensorMap ta, tb;
@@ -809,6 +809,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   if (kg2) {
     ok = make_map_3d(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 128, 2) &&
          make_map_3d(&tb, A, static_cast<uint64_t>(k), static_cast<uint64_t>(m), lda, static_cast<uint32_t>(b_rows), 2);
+    // (mc == 2: each stage's whole Bk half-box comes from one pair, so the box keeps b_rows rows)
   } else {
     if (!a_mn) ok = make_map(&ta, B, static_cast<uint64_t>(k), static_cast<uint64_t>(n), ldb, 64, 128);
     else ok = make_map(&ta, B, static_cast<uint64_t>(n), static_cast<uint64_t>(k), ldb, 64, 64);
@@ -867,7 +868,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   bool sk_used = false;
   const hgi::TcLaunch L = {&ta, &tb, &td, &p, dev, &di, cfg.max_ctas, skm_eff, &sk_used, stream};
   hgemm_status_t st;
-  if (kg2) st = hgi::dispatch_tc256_kg2(cg, f32, L);
+  if (kg2) st = hgi::dispatch_tc256_kg2(cg, f32, L, mc);
   else if (cg == 2 && bn == 512) st = hgi::dispatch_tc512(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L);
   else if (cg == 2)
     st = hgi::dispatch_tc256x2(mc, ag != nullptr, acc16, a_mn, b_mn, f32, L, g_env_direct != 0 && !tnf);

@@ -24,8 +24,15 @@ hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_m
   return dispatch_tc_layout<256, 2, 1>(a_mn, b_mn, f32, L);
 }
 
-hgemm_status_t dispatch_tc256_kg2(int cg, bool f32, const TcLaunch &L) {
+hgemm_status_t dispatch_tc256_kg2(int cg, bool f32, const TcLaunch &L, int mc) {
   if (cg != 2) return HGEMM_ERR_INVALID_VALUE;  // 1-SM 256-wide: two 96 KB stages only, not built
+#ifdef HGEMM_ENABLE_MC
+  if (mc == 2)
+    return f32 ? launch_tc<256, 2, false, false, true, 2, false, false, false, 2>(L)
+               : launch_tc<256, 2, false, false, false, 2, false, false, false, 2>(L);
+#else
+  (void)mc;
+#endif
   return f32 ? launch_tc<256, 2, false, false, true, 1, false, false, false, 2>(L)
              : launch_tc<256, 2, false, false, false, 1, false, false, false, 2>(L);
 }

@@ -59,7 +59,7 @@ hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_m
 hgemm_status_t dispatch_tc1(int bn, bool a_mn, bool b_mn, bool f32, const TcLaunch &L);
 // 256-wide CTA-pair tiles with k-group stages (KG = 2): TN layout,
 // K % 128 == 0, whole tiles; tensor maps are the 3-D k-group views (box {64, rows, 2})
-hgemm_status_t dispatch_tc256_kg2(int cg, bool f32, const TcLaunch &L);
+hgemm_status_t dispatch_tc256_kg2(int cg, bool f32, const TcLaunch &L, int mc = 1);
 hgemm_status_t dispatch_splitk64(int spl, bool a_mn, bool b_mn, bool f32, const CUtensorMap &ta,
                                  const CUtensorMap &tb, const hg::TcParams &p, int dev, cudaStream_t s,
                                  bool hm = false);

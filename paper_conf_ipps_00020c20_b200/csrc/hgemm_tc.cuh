@@ -473,7 +473,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT, KG>::THRE
                     const __grid_constant__ CUtensorMap tmD, const TcParams p) {
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ >= 1000)
   using S = TcShape<BN, CG, OUT_F32, EPI_DIRECT, KG>;
-  static_assert(KG == 1 || (KG == 2 && S::NH == 1 && !A_MN && !B_MN && MC == 1 && !AG),
+  static_assert(KG == 1 || (KG == 2 && S::NH == 1 && !A_MN && !B_MN && !AG),
                 "k-group stages: one accumulator half, K-major operands, whole tiles");
   constexpr int BM = S::BM;
   constexpr int BK = S::BK;
@@ -680,6 +680,14 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT, KG>::THRE
             const int h = half ? hsel : hh;
             const uint32_t sbh = sb + h * KG * B_HALF_BYTES;
             const int b_row = b_row0 + (half ? sub : h) * UMMA_N;
+            if constexpr (MC == 2 && KG == 2) {
+              // k-group stages: the whole Bk half-box of a stage (one 3-D box) is loaded by one
+              // pair, alternating per stage, and multicast to the same CTA position of both pairs
+              const uint16_t mc_mask = static_cast<uint16_t>((1u << prank) | (1u << (CG + prank)));
+              if ((((kb - wi.kb0) / KG) & 1) == static_cast<int>(pair))
+                tma_load_3d_pair_mc(&tmB, sbh, fb, 0, b_row, kb, mc_mask);
+              continue;
+            }
             if constexpr (MC == 2) {
               // this pair's share of the half-box, delivered to the same CTA position of both pairs
               const uint16_t mc_mask = static_cast<uint16_t>((1u << prank) | (1u << (CG + prank)));

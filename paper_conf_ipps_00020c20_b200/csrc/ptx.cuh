@@ -160,6 +160,16 @@ __device__ __forceinline__ void tma_load_3d_pair(const CUtensorMap *m, uint32_t 
       "l"(reinterpret_cast<uint64_t>(m)), "r"(bar_cluster), "r"(c0), "r"(c1), "r"(c2)
       : "memory");
 }
+// 3-D pair box multicast to the CTAs of `mask` (same offsets), completing on each destination
+// pair's leader mbarrier (experiments: 2-pair clusters with k-group stages).
+__device__ __forceinline__ void tma_load_3d_pair_mc(const CUtensorMap *m, uint32_t dst, uint32_t bar_cluster,
+                                                    int32_t c0, int32_t c1, int32_t c2, uint16_t mask) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster"
+      " [%0], [%1, {%3, %4, %5}], [%2], %6;" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(bar_cluster & 0xFEFFFFFFu), "r"(c0), "r"(c1), "r"(c2), "h"(mask)
+      : "memory");
+}
 __device__ __forceinline__ void tma_load_3d(const CUtensorMap *m, uint32_t dst, uint32_t bar, int32_t c0,
                                             int32_t c1, int32_t c2) {
   asm volatile(

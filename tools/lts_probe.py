@@ -3,7 +3,9 @@ persistent grid capped at fewer CTA pairs (each pair then runs several tiles in 
 a chip-wide L2-throughput limit lets the per-tile time fall as fewer SMs load, a per-SM
 limit keeps it (experiments; run under ncu for cold per-launch times).
 
-    python tools/lts_probe.py > order.txt
+    python tools/lts_probe.py [--warm] > order.txt
+
+--warm: no L2 flush between launches (run ncu with --cache-control none): operands L2-resident.
 """
 import os
 import sys
@@ -21,7 +23,8 @@ for (m, n, k) in [(4096, 1024, 4096), (2048, 2048, 8192)]:
     for mc in (0, 96, 64, 32, 16):
         binding.set_config("tc2", block_n=256, max_ctas=mc, stream_k=1)
         for _ in range(3):
-            w.zero_()
+            if "--warm" not in sys.argv:
+                w.zero_()
             binding.hgemm(m, n, k, 1.0, A, k, B, k, 0.0, C, m, "T", "N", "f16")
             torch.cuda.synchronize()
             print(f"{m}x{n}x{k} tc2/256 max_ctas={mc}", flush=True)
