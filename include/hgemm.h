@@ -147,7 +147,7 @@ typedef enum {
     HGEMM_KERNEL_SIMT = 1,       /* CUDA-core fallback (always available) */
     HGEMM_KERNEL_TC_1SM = 2,     /* tcgen05 cta_group::1, tile 128 x block_n */
     HGEMM_KERNEL_TC_2SM = 3,     /* tcgen05 cta_group::2 (CTA pair), tile 256 x block_n (256 or 512); 256-wide
-                                    tiles in layout TN with k % 128 == 0 and no stream-K load two k-blocks per
+                                    tiles in layout TN with k % 128 == 0 and n > 256 load two k-blocks per
                                     ring stage through 3-D TMA boxes (hgemm_get_last_config: splits = 2) */
     HGEMM_KERNEL_SPLITK = 4,     /* tcgen05 cta_group::1, tile 128 x block_n (64 or 128), K split over a
                                     cluster of `splits` CTAs, reduced through distributed shared memory */

@@ -69,7 +69,8 @@ const int g_env_sk_hm = env_int("HGEMM_SK_HM", 0);            // split-K 64-wide
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
 const bool g_env_flex = env_int("HGEMM_FLEX", 0) != 0;        // flexible tile widths in the automatic choice
 const int g_env_stream_a3d = env_int("HGEMM_STREAM_A3D", 1);  // streaming kernel: Ak through the 3-D k-group view
-const int g_env_tc_kg = env_int("HGEMM_TC_KG", 2);            // 256-wide tiles: k-blocks per ring stage (1 or 2)
+const int g_env_tc_kg = env_int("HGEMM_TC_KG", 2);
+const int g_env_tc_kg_sk = env_int("HGEMM_TC_KG_SK", 1);       // k-group stages also with stream-K (units of 2 k-blocks)            // 256-wide tiles: k-blocks per ring stage (1 or 2)
 const int g_env_direct = env_int("HGEMM_EPI_DIRECT", 0);      // 256-wide pair tiles: direct-store epilogue, 7 stages
 
 bool device_info(int dev, DeviceInfo &out) {
@@ -803,7 +804,7 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   const int64_t kg_tiles = cdiv(M, 256) * cdiv(N, 256);
   const bool kg2 = g_env_tc_kg == 2 && cg == 2 && bn == 256 && !a_mn && !b_mn && k % 128 == 0 && !tnf &&
                    !ag && !acc16 && !(cg == 2 && g_env_direct != 0) && M > 256 &&
-                   sk_plan(kg_tiles, di.num_sms / 2, cdiv(k, 64), skm & 15) < 0;
+                   (g_env_tc_kg_sk || sk_plan(kg_tiles, di.num_sms / 2, cdiv(k, 64), skm & 15) < 0);
   CUtensorMap ta, tb;
   bool ok;
   if (kg2) {

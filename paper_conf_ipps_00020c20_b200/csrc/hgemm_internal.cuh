@@ -138,14 +138,17 @@ hgemm_status_t launch_tc(const TcLaunch &L) {
   }
   t_half_used = half_tail;
   if (MC == 1 && !AG && !ACC16 && !half_tail) {
-    // k-group stages (KG = 2) run whole tiles only (work items of an even number of k-blocks)
-    const int dp = sk_plan(tiles, units, p.num_k_blocks, KG == 2 ? 1 : sk_mode);
+    // k-group stages (KG = 2): stream-K units of KG k-blocks, so every item starts and ends on
+    // a stage boundary
+    const int nku = p.num_k_blocks / KG;
+    const int dp = sk_plan(tiles, units, nku, sk_mode);
     float *ws = nullptr;
     int *flags = nullptr;
     if (dp >= 0 && units * CG * MC <= di.num_sms && sk_workspace(dev, L.stream, di.num_sms, &ws, &flags)) {
       p.dp_tiles = dp;
-      p.sk_u0 = static_cast<int64_t>(dp) * p.num_k_blocks;
-      p.sk_units = static_cast<int64_t>(tiles - dp) * p.num_k_blocks;
+      p.sk_kgu = KG;
+      p.sk_u0 = static_cast<int64_t>(dp) * nku;
+      p.sk_units = static_cast<int64_t>(tiles - dp) * nku;
       p.sk_ws = ws;
       p.sk_flags = flags;
       clusters = units;

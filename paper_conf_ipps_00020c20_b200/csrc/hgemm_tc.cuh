@@ -59,6 +59,7 @@ struct TcParams {
   // sk_units == 0: every tile whole (dp_tiles = all tiles).
   int32_t dp_tiles;
   int64_t sk_u0, sk_units;
+  int32_t sk_kgu;  // k-blocks per stream-K unit (KG = 2 stages: 2; 0/1 = one k-block)
   float *sk_ws;                      // one 128 x BN FP32 partial-accumulator slot per CTA
   int *sk_flags;                     // one flag per CTA: 1 = slot published; consumers reset it to 0
   // Fused all-gather of op(A) (hgemm_allgather_a, kernels with AG = true; DESIGN.md
@@ -114,21 +115,23 @@ __device__ __forceinline__ int64_t sk_begin(const TcParams &p, int c, int G) {
 // tile segments of its stream-K range in k order.  False past the last item.
 __device__ __forceinline__ bool get_item(const TcParams &p, int c, int G, int i, WorkItem &w) {
   const int n_dp = p.dp_tiles > c ? (p.dp_tiles - c + G - 1) / G : 0;
-  const int nkb = p.num_k_blocks;
   if (i < n_dp) {
     w.tile = c + i * G;
     w.kb0 = 0;
-    w.kb1 = nkb;
+    w.kb1 = p.num_k_blocks;
     return true;
   }
   if (p.sk_units == 0) return false;
+  // stream-K units are groups of sk_kgu k-blocks (k-group stages need even item bounds)
+  const int kgu = p.sk_kgu > 1 ? p.sk_kgu : 1;
+  const int nku = p.num_k_blocks / kgu;  // units per tile
   const int64_t u0 = sk_begin(p, c, G), u1 = sk_begin(p, c + 1, G);
-  const int t = static_cast<int>(u0 / nkb) + (i - n_dp);
-  const int64_t b = max(u0, static_cast<int64_t>(t) * nkb), e = min(u1, static_cast<int64_t>(t + 1) * nkb);
+  const int t = static_cast<int>(u0 / nku) + (i - n_dp);
+  const int64_t b = max(u0, static_cast<int64_t>(t) * nku), e = min(u1, static_cast<int64_t>(t + 1) * nku);
   if (b >= e) return false;
   w.tile = t;
-  w.kb0 = static_cast<int>(b - static_cast<int64_t>(t) * nkb);
-  w.kb1 = static_cast<int>(e - static_cast<int64_t>(t) * nkb);
+  w.kb0 = static_cast<int>(b - static_cast<int64_t>(t) * nku) * kgu;
+  w.kb1 = static_cast<int>(e - static_cast<int64_t>(t) * nku) * kgu;
   return true;
 }
 
@@ -949,7 +952,7 @@ __global__ void __launch_bounds__(TcShape<BN, CG, OUT_F32, EPI_DIRECT, KG>::THRE
       const int mode = wi.kb0 > 0 ? 1 : (wi.kb1 < p.num_k_blocks ? 2 : 0);
       int c_hi = cluster_id + 1;  // mode 2: clusters [cluster_id + 1, c_hi) hold this tile's partials
       if (mode == 2) {
-        const int64_t tile_end = static_cast<int64_t>(wi.tile + 1) * p.num_k_blocks;
+        const int64_t tile_end = static_cast<int64_t>(wi.tile + 1) * (p.num_k_blocks / (p.sk_kgu > 1 ? p.sk_kgu : 1));
         while (c_hi < num_clusters && sk_begin(p, c_hi, num_clusters) < tile_end) ++c_hi;
       }
       const int n_contrib = c_hi - cluster_id - 1;

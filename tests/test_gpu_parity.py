@@ -279,6 +279,32 @@ def test_stream_k_integer_exact(oracle_mod, kernel, bn, max_ctas):
     assert np.all(case.view(case.run_gpu()) == expect)
 
 
+@pytest.mark.parametrize("max_ctas", [8, 32])
+@pytest.mark.parametrize("out,beta", [("f16", 1.0), ("f32", 0.0)])
+def test_stream_k_kgroup(oracle_mod, max_ctas, out, beta):
+    """Stream-K with k-group stages (256-wide pair tiles, TN, k % 128 == 0): work items split at
+    even k-blocks (units of two), summed through the workspace in k order -- within tolerance,
+    deterministic across launches; integer inputs exact."""
+    from paper_conf_ipps_00020c20_b200 import binding
+    binding.set_config("tc2", block_n=256, max_ctas=max_ctas, stream_k=2)
+    m, n, k = 300, 520, 2048
+    C = inputs.uniform_f16(m, n, 7).astype(np.float32 if out == "f32" else np.float16)
+    case = GpuCase(inputs.uniform_f16(m, k, 5), inputs.uniform_f16(k, n, 6), "T", "N", 1.0, beta, C=C, out=out,
+                   pad=(8, 16, 8))
+    a, b, c = case.run_gpu(repeat=3)
+    assert case.stats["stream_k"] == 2 and case.stats["splits"] == 2, case.stats
+    u = np.uint32 if out == "f32" else np.uint16
+    assert np.array_equal(a.view(u), b.view(u)) and np.array_equal(a.view(u), c.view(u))
+    _, r, ab = case.oracle(oracle_mod)
+    assert_within_tolerance(case, a, r, ab)
+    opA, opB = inputs.integer_f16(m, k, 3, -4, 4), inputs.integer_f16(k, n, 4, -4, 4)
+    case = GpuCase(opA, opB, "T", "N", out="f32")
+    got = case.view(case.run_gpu())
+    assert case.stats["stream_k"] == 2 and case.stats["splits"] == 2, case.stats
+    _, r, _ = case.oracle(oracle_mod)
+    assert np.array_equal(got.astype(np.float64), r)
+
+
 def test_stream_k_graph_capture(oracle_mod):
     """Stream-K inside a captured CUDA graph: the workspace is created by an
     eager call on the stream first; replays reuse it (flags reset each launch)."""
