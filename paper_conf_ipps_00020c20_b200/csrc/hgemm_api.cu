@@ -505,6 +505,12 @@ void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, 
     double eff = (c.bn == 512 && beta_nonzero) ? (K < 4096 ? 0.90 : 0.97) : c.eff;
     // flexible tiles with beta != 0 take the chunked epilogue (C through registers)
     if (c.tn && beta_nonzero) eff *= 0.95;
+    // 1-SM tiles need 0.75-1 TMA box rows per tensor cycle (128 B each), far above what the
+    // TMA engine delivers (~0.3 rows/clk, profiles/r02/l2_ingest_study.log); short k loops hide
+    // it in the fixed costs, long ones do not: 1280 x 1280 x 5120 32.0 us with 128 x 128 tiles,
+    // 28.6 with CTA-pair 256-wide tiles + stream-K; 1536 x 1536 x 6144 37.2 vs 33.7 us
+    // (profiles/r02/chooser_probe.log)
+    if (c.cg == 1 && cdiv(K, 64) >= 64) eff *= 0.65;
     const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, width);
     const int64_t units = num_sms / c.cg;
     double waves = static_cast<double>(cdiv(tiles, units));
