@@ -69,8 +69,9 @@ const int g_env_sk_hm = env_int("HGEMM_SK_HM", 0);            // split-K 64-wide
 const int g_env_exp = env_int("HGEMM_EXP", 0);                // TcParams::exp_flags
 const bool g_env_flex = env_int("HGEMM_FLEX", 0) != 0;        // flexible tile widths in the automatic choice
 const int g_env_stream_a3d = env_int("HGEMM_STREAM_A3D", 1);  // streaming kernel: Ak through the 3-D k-group view
-const int g_env_tc_kg = env_int("HGEMM_TC_KG", 2);
-const int g_env_tc_kg_sk = env_int("HGEMM_TC_KG_SK", 1);       // k-group stages also with stream-K (units of 2 k-blocks)            // 256-wide tiles: k-blocks per ring stage (1 or 2)
+const int g_env_tc_kg = env_int("HGEMM_TC_KG", 2);            // 256-wide pair / 128 x 128 tiles: k-blocks per ring stage (1 or 2)
+const int g_env_tc_kg_sk = env_int("HGEMM_TC_KG_SK", 1);      // k-group stages also with stream-K (units of 2 k-blocks)
+const int g_env_tc1_kg = env_int("HGEMM_TC1_KG", 1);          // k-group stages for 1-SM 128 x 128 tiles too
 const int g_env_direct = env_int("HGEMM_EPI_DIRECT", 0);      // 256-wide pair tiles: direct-store epilogue, 7 stages
 
 bool device_info(int dev, DeviceInfo &out) {
@@ -483,7 +484,7 @@ inline double flex_eff(int tn) {
 // 256-wide CTA-pair kernel may use a flexible tile width (K-major Bk); tn returns the
 // chosen width (0: the kernel's own BN).
 void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, int forced_cg, int sk_mode, int &cg,
-               int &bn, bool flex_ok, int &tn) {
+               int &bn, bool flex_ok, int &tn, bool kg_ok) {
   struct Cand { int cg, bn, tn; double eff; };
   // eff: relative per-SM throughput of the tile shape.  Larger tiles move
   // fewer L2->SMEM bytes per FLOP (pair 256x512: 171 FLOP/B, 256x256: 128,
@@ -505,12 +506,13 @@ void choose_tc(int64_t M, int64_t N, int64_t K, bool beta_nonzero, int num_sms, 
     double eff = (c.bn == 512 && beta_nonzero) ? (K < 4096 ? 0.90 : 0.97) : c.eff;
     // flexible tiles with beta != 0 take the chunked epilogue (C through registers)
     if (c.tn && beta_nonzero) eff *= 0.95;
-    // 1-SM tiles need 0.75-1 TMA box rows per tensor cycle (128 B each), far above what the
-    // TMA engine delivers (~0.3 rows/clk, profiles/r02/l2_ingest_study.log); short k loops hide
-    // it in the fixed costs, long ones do not: 1280 x 1280 x 5120 32.0 us with 128 x 128 tiles,
-    // 28.6 with CTA-pair 256-wide tiles + stream-K; 1536 x 1536 x 6144 37.2 vs 33.7 us
-    // (profiles/r02/chooser_probe.log)
-    if (c.cg == 1 && cdiv(K, 64) >= 64) eff *= 0.65;
+    // 1-SM tiles with one k-block per stage need 0.75-1 TMA box rows per tensor cycle (128 B
+    // each), far above what the TMA engine delivers (~0.3 rows/clk, profiles/r02/
+    // l2_ingest_study.log); short k loops hide it in the fixed costs, long ones do not:
+    // 1280 x 1280 x 5120 34.1 us with 128 x 128 tiles, 28.6 with CTA-pair 256-wide tiles +
+    // stream-K.  The 128 x 128 tile with k-group stages (kg_ok: layout TN, k % 128 == 0) halves
+    // its rows per cycle and beats both there (26.8 us; profiles/r02/chooser_probe.log).
+    if (c.cg == 1 && cdiv(K, 64) >= 64 && !(kg_ok && c.bn == 128)) eff *= 0.65;
     const int64_t tiles = cdiv(M, 128 * c.cg) * cdiv(N, width);
     const int64_t units = num_sms / c.cg;
     double waves = static_cast<double>(cdiv(tiles, units));
@@ -786,7 +788,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
     // flexible widths are never chosen automatically: measured slower than the 256-wide tile
     // (with stream-K) at every mid-size shape tried (profiles/r02/flex_tile_sweep.log; DESIGN.md
     // "Flexible tile width"); the candidates stay available to the model for experiments
-    choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, skm, cg, bn, flex_ok && g_env_flex, tnf);
+    choose_tc(M, N, k, beta != 0.0f, di.num_sms, forced_cg, skm, cg, bn, flex_ok && g_env_flex, tnf,
+              g_env_tc_kg == 2 && g_env_tc1_kg && !a_mn && !b_mn && k % 128 == 0 && M > 256 && !ag && !acc16);
   }
   const int skm_eff = tnf ? ((skm & ~15) | 1) : skm;  // flexible tiles: whole tiles, no stream-K
   const int b_rows = (tnf ? tnf : (bn > 256 ? 256 : bn)) / cg;  // Bk rows per CTA per accumulator half
@@ -808,7 +811,8 @@ hgemm_status_t hgemm_core(int64_t m, int64_t n, int64_t k, float alpha, const vo
   // HBM-streaming case, where 3 stages of 64 KB keep fewer bytes in flight than 6 of 32 KB);
   // profiles/r02/tc_kgroup_ab.log.
   const int64_t kg_tiles = cdiv(M, 256) * cdiv(N, 256);
-  const bool kg2 = g_env_tc_kg == 2 && cg == 2 && bn == 256 && !a_mn && !b_mn && k % 128 == 0 && !tnf &&
+  const bool kg2 = g_env_tc_kg == 2 && ((cg == 2 && bn == 256) || (cg == 1 && bn == 128 && g_env_tc1_kg)) &&
+                   !a_mn && !b_mn && k % 128 == 0 && !tnf &&
                    !ag && !acc16 && !(cg == 2 && g_env_direct != 0) && M > 256 &&
                    (g_env_tc_kg_sk || sk_plan(kg_tiles, di.num_sms / 2, cdiv(k, 64), skm & 15) < 0);
   CUtensorMap ta, tb;

@@ -25,7 +25,10 @@ hgemm_status_t dispatch_tc256x2(int mc, bool ag, bool acc16, bool a_mn, bool b_m
 }
 
 hgemm_status_t dispatch_tc256_kg2(int cg, bool f32, const TcLaunch &L, int mc) {
-  if (cg != 2) return HGEMM_ERR_INVALID_VALUE;  // 1-SM 256-wide: two 96 KB stages only, not built
+  // 1-SM 128 x 128 tiles: three 64 KB stages, like the CTA-pair 256-wide tile (the 1-SM
+  // 256-wide tile would have two 96 KB stages only: not built)
+  if (cg == 1) return f32 ? launch_tc<128, 1, false, false, true, 1, false, false, false, 2>(L)
+                          : launch_tc<128, 1, false, false, false, 1, false, false, false, 2>(L);
 #ifdef HGEMM_ENABLE_MC
   if (mc == 2)
     return f32 ? launch_tc<256, 2, false, false, true, 2, false, false, false, 2>(L)

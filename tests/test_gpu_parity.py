@@ -279,14 +279,14 @@ def test_stream_k_integer_exact(oracle_mod, kernel, bn, max_ctas):
     assert np.all(case.view(case.run_gpu()) == expect)
 
 
-@pytest.mark.parametrize("max_ctas", [8, 32])
+@pytest.mark.parametrize("kernel,bn,max_ctas", [("tc2", 256, 8), ("tc2", 256, 32), ("tc1", 128, 12)])
 @pytest.mark.parametrize("out,beta", [("f16", 1.0), ("f32", 0.0)])
-def test_stream_k_kgroup(oracle_mod, max_ctas, out, beta):
+def test_stream_k_kgroup(oracle_mod, kernel, bn, max_ctas, out, beta):
     """Stream-K with k-group stages (256-wide pair tiles, TN, k % 128 == 0): work items split at
     even k-blocks (units of two), summed through the workspace in k order -- within tolerance,
     deterministic across launches; integer inputs exact."""
     from paper_conf_ipps_00020c20_b200 import binding
-    binding.set_config("tc2", block_n=256, max_ctas=max_ctas, stream_k=2)
+    binding.set_config(kernel, block_n=bn, max_ctas=max_ctas, stream_k=2)
     m, n, k = 300, 520, 2048
     C = inputs.uniform_f16(m, n, 7).astype(np.float32 if out == "f32" else np.float16)
     case = GpuCase(inputs.uniform_f16(m, k, 5), inputs.uniform_f16(k, n, 6), "T", "N", 1.0, beta, C=C, out=out,
@@ -399,15 +399,16 @@ def test_splitk_auto_small_problems(oracle_mod, w, tA, tB, out, spl):
             assert_within_tolerance(case, got, r, ab)
 
 
+@pytest.mark.parametrize("kernel,bn", [("tc2", 256), ("tc1", 128)])
 @pytest.mark.parametrize("m,n,k", [(520, 600, 1024), (300, 1100, 384), (1000, 700, 2048)])
 @pytest.mark.parametrize("out", ["f16", "f32"])
 @pytest.mark.parametrize("beta", [0.0, 1.0])
-def test_tc_kgroup_stages(oracle_mod, m, n, k, out, beta):
-    """256-wide CTA-pair tiles with two k-blocks per ring stage (3-D TMA boxes; layout TN,
-    k % 128 == 0, stream-K off): random inputs within the BJ bound, integer inputs bit-exact,
-    ragged m / n."""
+def test_tc_kgroup_stages(oracle_mod, kernel, bn, m, n, k, out, beta):
+    """256-wide CTA-pair tiles and 1-SM 128 x 128 tiles with two k-blocks per ring stage (3-D
+    TMA boxes; layout TN, k % 128 == 0, stream-K off): random inputs within the BJ bound,
+    integer inputs bit-exact, ragged m / n."""
     from paper_conf_ipps_00020c20_b200 import binding
-    binding.set_config("tc2", block_n=256, stream_k=1)
+    binding.set_config(kernel, block_n=bn, stream_k=1)
     for integer in (False, True):
         if integer:
             opA, opB = inputs.integer_f16(m, k, 21, -2, 2), inputs.integer_f16(k, n, 22, -2, 2)
@@ -416,7 +417,7 @@ def test_tc_kgroup_stages(oracle_mod, m, n, k, out, beta):
             opA, opB, C = inputs.uniform_f16(m, k, 21), inputs.uniform_f16(k, n, 22), inputs.uniform_f16(m, n, 23)
         case = GpuCase(opA, opB, "T", "N", 1.0, beta, C=C, out=out)
         got = case.run_gpu()
-        assert case.stats["last_kernel"] == "tc2" and case.stats["block_n"] == 256, case.stats
+        assert case.stats["last_kernel"] == kernel and case.stats["block_n"] == bn, case.stats
         assert case.stats["splits"] == 2, case.stats   # k-group stages
         c_ref, r, ab = case.oracle(oracle_mod)
         if integer:
