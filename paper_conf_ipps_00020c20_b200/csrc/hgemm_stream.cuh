@@ -347,6 +347,13 @@ __global__ void __launch_bounds__(192, 1)
   tc_fence_before();
   __syncthreads();
   if (threadIdx.x == 0) ST_TRACE(6);
+#ifdef HGEMM_TRACE
+  if (threadIdx.x == 0 && p.probe != nullptr) {  // slot 7: the SM this CTA ran on
+    uint32_t smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    p.probe[8 * blockIdx.x + 7] = smid;
+  }
+#endif
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc<1>(tmem_base, 512);
